@@ -1,0 +1,344 @@
+#!/usr/bin/env python
+"""bench.py -- model-update latency of the Viper hot path on B200.
+
+Default (N=1): BASELINE.json configs[0], the only single-GPU configuration:
+PtychoNN-sized fp32 model (40 tensors, 4.6 MB), 1 producer -> 1 consumer on
+one GPU (in-process loopback, GPU tier, SYNC mode).  One step = one versioned
+model update: pack + seal (K2) -> publish/notify -> install + verify (K6) ->
+device-side atomic version swap; publish() returns once the consumer serves v.
+
+Timing: per step, L2 is flushed (a 256 MiB write, > the 126 MB L2) and the
+producer's tensors are rewritten with VGEN(v) (the synthetic "optimizer step")
+OUTSIDE the timed interval; each update is timed with CUDA events on the
+publishing stream (start before publish, end after it returned) and with the
+host clock (publish entry -> return = the swap is visible).  value = mean
+device-event latency over the K timed steps.
+
+Extra keys: roofline of the dominant kernel (library-recorded CUDA events,
+VIPER_FLAG_TIMING), cpu_baseline (the oracle on host cores), e2e (host
+buffers: H2D of the new weights + publish + D2H of the seal digest), clocks,
+gpu_launches, and a 1-GPU loopback sweep over the other BASELINE.json model
+sizes (not the headline).
+
+--impl reference: the oracle (plain C, oracle/) on the host cores, same
+config/metric -- the deliberately slow reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "model-update latency (ms) and GB/s vs NVLink/HBM roofline at 1->1/3/7 GPUs"
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 6:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ---------------------------------------------------------------- GPU arm
+def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tier=None, timing=True):
+    """Producer + 1 consumer on this GPU; returns per-step timings + stats."""
+    import torch
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    prod_t = G.alloc_model(specs)
+    cons_t = G.alloc_model(specs)
+    mname = f"bench-{name}-{os.getpid()}-{time.monotonic_ns()}"
+    flags = V.FLAG_TIMING if timing else 0
+    mode = V.SYNC if mode is None else mode
+    tier = V.TIER_GPU if tier is None else tier
+    cons = V.Model(mname, V.CONSUMER, cons_t, flags=flags, tier=tier)
+    prod = V.Model(mname, V.PRODUCER, prod_t, flags=flags, mode=mode, tier=tier)
+    st = torch.cuda.current_stream()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    dev_ms, host_ms, pack_us, inst_us = [], [], [], []
+    try:
+        for i in range(warmup + steps):
+            v = i + 1
+            G.fill_model(prod_t, specs, seed, v, stream=st)
+            G.l2_flush(flush_buf, stream=st)
+            torch.cuda.synchronize()
+            ev0.record(st)
+            t0 = time.perf_counter()
+            prod.publish(v, stream=st)
+            t1 = time.perf_counter()
+            ev1.record(st)
+            ev1.synchronize()
+            if i >= warmup:
+                dev_ms.append(ev0.elapsed_time(ev1))
+                host_ms.append((t1 - t0) * 1e3)
+                pack_us.append(prod.stats()["t_pack_dev_us"])
+                inst_us.append(cons.stats()["t_install_dev_us"])
+        view = cons.acquire_latest()
+        ok = view.version == warmup + steps and all(
+            torch.equal(g.view(torch.uint8), p.view(torch.uint8)) for g, p in zip(view.tensors(cons_t), prod_t))
+        cons.release(view)
+        s_packed = prod.stats()["s_packed"]
+        nchunks = prod.stats()["nchunks"]
+    finally:
+        cons.close()
+        prod.close()
+    return {"dev_ms": dev_ms, "host_ms": host_ms, "pack_us": pack_us, "install_us": inst_us, "ok": ok,
+            "s_packed": s_packed, "nchunks": nchunks, "bytes": synth.model_bytes(name), "tensors": len(specs)}
+
+
+def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
+    """Same update through the public API with HOST buffers: each step copies
+    the new weights from pinned host memory (H2D), publishes, and reads the
+    seal digest back (D2H)."""
+    import torch
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    prod_t = G.alloc_model(specs)
+    cons_t = G.alloc_model(specs)
+    host = []
+    for i in range(2):  # two host versions, alternated
+        tmp = G.alloc_model(specs)
+        G.fill_model(tmp, specs, seed, 1000 + i)
+        host.append([t.cpu().pin_memory() for t in tmp])
+        del tmp
+    mname = f"e2e-{name}-{os.getpid()}-{time.monotonic_ns()}"
+    cons = V.Model(mname, V.CONSUMER, cons_t)
+    prod = V.Model(mname, V.PRODUCER, prod_t)
+    st = torch.cuda.current_stream()
+    _, seals_ptr, nchunks = prod.debug_buffers()
+    digest = torch.empty(2 * nchunks, dtype=torch.int64).pin_memory()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    times = []
+    h2d = sum(t.numel() * t.element_size() for t in host[0])
+    try:
+        for i in range(warmup + steps):
+            G.l2_flush(flush_buf, stream=st)
+            torch.cuda.synchronize()
+            ev0.record(st)
+            for d, h in zip(prod_t, host[i % 2]):
+                d.copy_(h, non_blocking=True)
+            prod.publish(i + 1, stream=st)
+            _, seals_ptr, _ = prod.debug_buffers()
+            like = torch.empty(4 * nchunks, dtype=torch.int32, device="cuda")
+            digest.copy_(V._from_ptr(seals_ptr, like).view(torch.int64), non_blocking=True)
+            ev1.record(st)
+            ev1.synchronize()
+            if i >= warmup:
+                times.append(ev0.elapsed_time(ev1))
+    finally:
+        cons.close()
+        prod.close()
+    return {"ms": statistics.mean(times), "h2d": h2d, "d2h": digest.numel() * 8}
+
+
+def cpu_baseline(synth, name, budget_s=10.0, max_updates=400):
+    """The oracle (plain C, single thread, as it stands) timed on this host's
+    cores on a bounded sample: repeated updates of the same config."""
+    from oracle import transfer as T
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    nb = [synth.nbytes_of(s) for s in specs]
+    versions = [[synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)] for v in (1, 2)]
+    c = T.Consumer(nb)
+    p = T.Producer(nb, [c])
+    times = []
+    t_start = time.perf_counter()
+    v = 0
+    try:
+        while time.perf_counter() - t_start < budget_s and len(times) < max_updates:
+            v += 1
+            t0 = time.perf_counter()
+            st = p.publish(v, versions[v % 2])
+            times.append((time.perf_counter() - t0) * 1e3)
+            assert st == T.OK
+    finally:
+        p.close()
+        c.close()
+    return {"value": statistics.mean(times), "unit": "ms", "cores": 1, "kind": "oracle",
+            "sample": f"{len(times)} oracle updates of {name} (pack+seal+deliver+verify+install+swap, 1 consumer)"}
+
+
+def gpu_arm(args):
+    import torch
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    import synth
+    from synth import gpu as G
+    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    name = args.config
+    peak, peak_kind = load_peaks()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    # ---- headline
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        r = run_update_bench(V, G, synth, name, args.steps, args.warmup, flush)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    mean_ms = statistics.mean(r["dev_ms"])
+    if world > 1:
+        t = torch.tensor([mean_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        mean_ms = float(t.item())
+    pack = statistics.median(r["pack_us"])
+    inst = statistics.median(r["install_us"])
+    alg = 2 * r["bytes"]
+    dom, dom_us = ("pack_seal", pack) if pack >= inst else ("install_verify", inst)
+    achieved = alg / (dom_us * 1e-6) / 1e9
+    out = {
+        "metric": METRIC, "value": round(mean_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(mean_ms, 6), "higher_is_better": False,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+        "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
+        "config": {"workload": f"{name}: 1 producer -> 1 consumer, 1 GPU loopback (BASELINE.json configs[0])"
+                   if name == "ptychonn" else f"{name} 1-GPU loopback",
+                   "tensors": r["tensors"], "model_bytes": r["bytes"], "packed_bytes": r["s_packed"],
+                   "tier": "gpu", "mode": "sync", "l2": "flushed (256 MiB write) before every timed update",
+                   "parallelism": "replicas" if world > 1 else "single GPU"},
+        "update_gbps": round(r["bytes"] / (mean_ms * 1e-3) / 1e9, 3),
+        "host_latency_ms": round(statistics.mean(r["host_ms"]), 6),
+        "latency_p50_ms": round(statistics.median(r["dev_ms"]), 6),
+        "latency_min_ms": round(min(r["dev_ms"]), 6),
+        "kernels_us": {"pack_seal": round(pack, 3), "install_verify": round(inst, 3)},
+        "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 2), "peak": peak,
+                     "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": None,
+                     "peak_kind": peak_kind, "algorithmic_bytes": alg},
+        "parity_ok": r["ok"],
+        "gpu_launches": 2 * args.steps,
+    }
+    out["clocks"] = clk.summary()
+    if rank == 0:
+        e = run_e2e(V, G, synth, name, max(3, args.steps // 2), args.warmup, flush)
+        out["e2e"] = {"value": round(e["ms"], 6), "unit": "ms", "h2d_bytes_per_step": e["h2d"],
+                      "d2h_bytes_per_step": e["d2h"]}
+        if not args.no_sweep:
+            sweep = {}
+            for nm in ["resnet50", "vit_b16", "gpt2_xl", "llama3_8b"]:
+                if nm == name:
+                    continue
+                try:
+                    s = run_update_bench(V, G, synth, nm, 5, 3, flush)
+                    pk, ins = statistics.median(s["pack_us"]), statistics.median(s["install_us"])
+                    lat = statistics.mean(s["dev_ms"])
+                    sweep[nm] = {"latency_ms": round(lat, 4), "pack_us": round(pk, 2), "install_us": round(ins, 2),
+                                 "pack_hbm_frac": round(2 * s["bytes"] / (pk * 1e-6) / 1e9 / peak, 4),
+                                 "install_hbm_frac": round(2 * s["bytes"] / (ins * 1e-6) / 1e9 / peak, 4),
+                                 "update_gbps": round(s["bytes"] / (lat * 1e-3) / 1e9, 2), "parity_ok": s["ok"]}
+                except Exception as ex:  # report, never hide
+                    sweep[nm] = {"error": str(ex)[:200]}
+                torch.cuda.empty_cache()
+            out["loopback_sweep"] = sweep
+        out["cpu_baseline"] = cpu_baseline(synth, name, budget_s=args.cpu_budget)
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def reference_arm(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import synth
+    name = args.config
+    res = []
+    for i in range(args.warmup + args.steps):
+        cb = cpu_baseline(synth, name, budget_s=max(1.0, args.cpu_budget / max(args.steps, 1)), max_updates=20)
+        if i >= args.warmup:
+            res.append(cb["value"])
+    v = statistics.mean(res)
+    out = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "ms", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(v, 4), "higher_is_better": False,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+           "data": "synthetic (VGEN)", "config": {"workload": f"{name}: oracle update on host cores"},
+           "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": 1, "kind": "oracle",
+                            "sample": "each step = up to 20 oracle updates, mean ms per update"},
+           "e2e": {"value": round(v, 4), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="viper", choices=["viper", "reference"])
+    ap.add_argument("--config", default="ptychonn", choices=["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
+    ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=10.0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        reference_arm(args)
+    else:
+        gpu_arm(args)
+
+
+if __name__ == "__main__":
+    main()

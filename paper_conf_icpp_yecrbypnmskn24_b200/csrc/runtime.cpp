@@ -1,0 +1,850 @@
+// runtime.cpp -- the Model Weights Handler (PAPER.md s4.4 P:1671-1800, Fig. 7)
+// rebuilt for one process per B200: registration / manifest,
+// publish = snapshot + notify, the consumer's update thread that
+// installs into the alternative copy and swaps atomically (P:1214-1227,
+// P:1424-1428), and the reader-side acquire/release.
+//
+// Every byte moves in the kernels of kernels.cu; this file only decides what
+// to launch, when, and on which stream.  There is no CPU data path.
+#include "runtime.h"
+
+#include <linux/futex.h>
+#include <sched.h>
+#include <sys/syscall.h>
+#include <time.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+namespace vp {
+
+static thread_local std::string t_err;
+
+viper_status set_error(viper_status st, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    t_err = buf;
+    return st;
+}
+
+#define CUDA_TRY(x)                                                                                  \
+    do {                                                                                             \
+        cudaError_t e_ = (x);                                                                        \
+        if (e_ != cudaSuccess)                                                                       \
+            return set_error(VIPER_E_CUDA, "%s failed: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, \
+                             __LINE__);                                                              \
+    } while (0)
+
+int64_t now_ns() {
+    timespec ts;
+    clock_gettime(CLOCK_MONOTONIC, &ts);
+    return (int64_t)ts.tv_sec * 1000000000ll + ts.tv_nsec;
+}
+
+// Shared (non-private) futexes: they also work on words in a shm segment.
+void futex_wake_all(std::atomic<uint32_t> *w) {
+    syscall(SYS_futex, reinterpret_cast<uint32_t *>(w), FUTEX_WAKE, INT_MAX, nullptr, nullptr, 0);
+}
+
+void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us) {
+    timespec ts, *tp = nullptr;
+    if (timeout_us >= 0) {
+        ts.tv_sec = timeout_us / 1000000;
+        ts.tv_nsec = (timeout_us % 1000000) * 1000;
+        tp = &ts;
+    }
+    syscall(SYS_futex, reinterpret_cast<uint32_t *>(w), FUTEX_WAIT, expected, tp, nullptr, 0);
+}
+
+static inline void cpu_relax() { __builtin_ia32_pause(); }
+
+// ------------------------------------------------------------------ manifest
+// LAY (R16) + the warp work list.  Items never cross a seal chunk
+// and are at most item_max bytes; splits fall on 16-B multiples of the tensor.
+static viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes,
+                                   uint32_t align, int device) {
+    m.n = n;
+    m.nbytes.resize(n);
+    m.offsets.resize(n);
+    m.chunk_bytes = chunk_bytes;
+    m.align = align;
+    uint64_t off = 0;
+    for (int32_t i = 0; i < n; i++) {
+        m.nbytes[i] = t[i].nbytes;
+        m.offsets[i] = off;
+        off = (off + t[i].nbytes + align - 1) / align * align;
+    }
+    m.s_packed = off;
+    m.nchunks = (uint32_t)((m.s_packed + chunk_bytes - 1) / chunk_bytes);
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    // item size: enough items for ~4 per resident warp, 2 KiB .. 64 KiB, 512-B multiple
+    uint64_t target = m.s_packed / ((uint64_t)sms * 32 * 4) + 1;
+    uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), 65536);
+    if (item_max > chunk_bytes) item_max = chunk_bytes;
+    m.items.clear();
+    std::vector<uint32_t> per_chunk(m.nchunks, 0);
+    for (int32_t i = 0; i < n; i++) {
+        uint64_t done = 0;
+        while (done < m.nbytes[i]) {
+            uint64_t p = m.offsets[i] + done;
+            uint64_t chunk = p / chunk_bytes;
+            uint64_t chunk_end = (chunk + 1) * chunk_bytes;
+            uint64_t len = std::min<uint64_t>({item_max, m.nbytes[i] - done, chunk_end - p});
+            Item it{};
+            it.packed_off = p;
+            it.tensor_off = done;
+            it.nbytes = (uint32_t)len;
+            it.tensor = (uint32_t)i;
+            it.chunk = (uint32_t)chunk;
+            m.items.push_back(it);
+            per_chunk[chunk]++;
+            done += len;
+        }
+    }
+    for (uint32_t c = 0; c < m.nchunks; c++)
+        if (per_chunk[c] == 0) return set_error(VIPER_E_INVAL, "chunk %u has no data (align > chunk?)", c);
+    for (auto &it : m.items) it.chunk_items = per_chunk[it.chunk];
+    if (m.items.size() >= (size_t)UINT32_MAX) return set_error(VIPER_E_INVAL, "too many work items");
+    if (!m.items.empty()) {
+        CUDA_TRY(cudaMalloc(&m.d_items, m.items.size() * sizeof(Item)));
+        CUDA_TRY(cudaMemcpy(m.d_items, m.items.data(), m.items.size() * sizeof(Item), cudaMemcpyHostToDevice));
+    }
+    return VIPER_OK;
+}
+
+static viper_status alloc_scratch(viper_model *m) {
+    const size_t nch = m->man.nchunks ? m->man.nchunks : 1;
+    const size_t bytes = nch * sizeof(uint64_t) + nch * sizeof(uint32_t) + 64;
+    CUDA_TRY(cudaMalloc(&m->scratch_alloc, bytes));
+    CUDA_TRY(cudaMemset(m->scratch_alloc, 0, bytes));
+    uint8_t *p = (uint8_t *)m->scratch_alloc;
+    m->scratch.acc = (uint64_t *)p;
+    m->scratch.cnt = (uint32_t *)(p + nch * sizeof(uint64_t));
+    m->scratch.done = (uint32_t *)(p + nch * sizeof(uint64_t) + nch * sizeof(uint32_t));
+    m->scratch.err = m->scratch.done + 4;
+    return VIPER_OK;
+}
+
+// ------------------------------------------------------- in-process registry
+static std::mutex g_reg_mu;
+static std::map<std::string, Channel *> g_reg;
+
+static viper_status channel_open(const std::string &name, const Manifest &man, Channel **out) {
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    auto it = g_reg.find(name);
+    Channel *ch;
+    if (it == g_reg.end()) {
+        ch = new Channel();
+        ch->name = name;
+        ch->nbytes = man.nbytes;
+        void *p = nullptr;
+        CUDA_TRY(cudaHostAlloc(&p, sizeof(Ctrl), cudaHostAllocMapped | cudaHostAllocPortable));
+        memset(p, 0, sizeof(Ctrl));
+        ch->ctrl = new (p) Ctrl();
+        ch->ctrl->magic = kCtrlMagic;
+        void *d = nullptr;
+        CUDA_TRY(cudaHostGetDevicePointer(&d, p, 0));
+        ch->ctrl_dev = (Ctrl *)d;
+        g_reg[name] = ch;
+    } else {
+        ch = it->second;
+        if (ch->nbytes != man.nbytes)
+            return set_error(VIPER_E_INVAL, "model '%s': tensor list differs from the other endpoints", name.c_str());
+    }
+    ch->refs++;
+    *out = ch;
+    return VIPER_OK;
+}
+
+static void channel_close(Channel *ch) {
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    if (--ch->refs > 0) return;
+    g_reg.erase(ch->name);
+    cudaFreeHost(ch->ctrl);
+    delete ch;
+}
+
+// --------------------------------------------------------------- install path
+static void fire_callback(viper_model *c, uint64_t v, viper_status st) {
+    void (*cb)(uint64_t, viper_status, void *);
+    void *user;
+    {
+        std::lock_guard<std::mutex> lk(c->cb_mu);
+        cb = c->cb;
+        user = c->cb_user;
+    }
+    if (cb) cb(v, st, user);
+}
+
+// Pin the latest published snapshot (Dekker pair with the producer's
+// pub_state store -> pin scan).  Returns false when
+// nothing is published.
+static bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
+    for (;;) {
+        const uint64_t ps = ctrl->pub_state.load();
+        if (ps == 0) return false;
+        r->pin.store(ps >> 1);
+        if (ctrl->pub_state.load() == ps) {
+            *v = ps >> 1;
+            *b = (int)(ps & 1);
+            return true;
+        }
+        r->pin.store(0);
+    }
+}
+
+// Enqueue the install of snapshot slot b (version v) of producer p into the
+// inactive slot of consumer c on stream st.  Caller holds c->install_mu and
+// has pinned v.  wait_ready: make st wait for the producer's snapshot event.
+static viper_status enqueue_install(viper_model *c, viper_model *p, uint64_t v, int b, cudaStream_t st,
+                                    bool wait_ready) {
+    ConsRec *r = c->rec;
+    const uint64_t cur = r->state.load();
+    const int target = cur == 0 ? 0 : (int)(1 - (cur & 1));
+    // The alternative copy is written only when no reader pins it (a7).
+    const int64_t t0 = now_ns();
+    while (r->ref[target].load() != 0) {
+        if (now_ns() - t0 > 10ll * 1000000000ll)
+            return set_error(VIPER_E_TIMEOUT, "readers kept slot %d pinned for 10 s", target);
+        sched_yield();
+    }
+    const double waited = (now_ns() - t0) / 1e3;
+    const uint8_t *src;
+    const Seal *seals;
+    if (wait_ready) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
+    if (c->cfg.tier == VIPER_TIER_DRAM) {
+        // Host-to-Host channel: host staging -> this GPU's staging
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, p->h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage_seals, p->h_seal[b], sizeof(Seal) * c->man.nchunks,
+                                 cudaMemcpyHostToDevice, st));
+        src = c->d_stage;
+        seals = c->d_stage_seals;
+    } else {
+        src = p->d_snap[b];
+        seals = p->d_seal[b];
+    }
+    InstallArgs a{};
+    a.items = c->man.d_items;
+    a.nitems = (uint32_t)c->man.items.size();
+    a.nchunks = c->man.nchunks;
+    a.dst = c->d_slot[target];
+    a.packed = src;
+    a.seals = seals;
+    a.s = c->scratch;
+    a.version = v;
+    a.target = (uint32_t)target;
+    a.fault_item = ~0u;
+    if (c->fault_next.exchange(false) && a.nitems) a.fault_item = a.nitems / 2;
+    a.status_h = (volatile int32_t *)&c->rec_dev->status;
+    a.pin_h = (volatile uint64_t *)&c->rec_dev->pin;
+    a.state_h = (volatile uint64_t *)&c->rec_dev->state;
+    r->status.store(1);  // "in flight"
+    const bool timing = c->cfg.flags & VIPER_FLAG_TIMING;
+    if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
+    CUDA_TRY(launch_install(a, c->geo, st));
+    if (timing) {
+        CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
+        c->timing_pending = true;
+    }
+    {
+        std::lock_guard<std::mutex> lk(c->stats_mu);
+        c->stats.writer_wait_us = waited;
+    }
+    return VIPER_OK;
+}
+
+// After the install kernel of v completed on the host's view of the stream.
+static viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
+    ConsRec *r = c->rec;
+    viper_status st = r->status.load();
+    if (st == 1) st = set_error(VIPER_E_CUDA, "install kernel did not report");
+    float dev_ms = -1.f;
+    if (c->timing_pending && cudaEventElapsedTime(&dev_ms, c->ev_t[0], c->ev_t[1]) == cudaSuccess)
+        c->timing_pending = false;
+    {
+        std::lock_guard<std::mutex> lk(c->stats_mu);
+        if (dev_ms >= 0) c->stats.t_install_dev_us = dev_ms * 1e3;
+        c->stats.last_status = st;
+        c->stats.t_install_us = t_install_us;
+        if (st == VIPER_OK) {
+            c->stats.installs++;
+            c->stats.version = v;
+        } else {
+            c->stats.failures++;
+        }
+    }
+    r->pin.store(0);
+    r->last_status.store(st);
+    r->done_version.store(v);
+    r->done_seq.fetch_add(1);
+    futex_wake_all(&r->done_seq);
+    return st;
+}
+
+static void update_loop(viper_model *c) {
+    cudaSetDevice(c->device);
+    Ctrl *ctrl = c->ctrl;
+    ConsRec *r = c->rec;
+    while (!c->stop.load()) {
+        const uint32_t seq = ctrl->pub_seq.load();
+        const uint64_t ps = ctrl->pub_state.load();
+        bool work;
+        {
+            // SYNC producers install inline; the thread only catches a consumer
+            // up that registered after the last publish.
+            std::lock_guard<std::mutex> lk(c->install_mu);
+            viper_model *p = c->chan ? c->chan->producer : nullptr;
+            const bool async = p && p->cfg.mode == VIPER_ASYNC;
+            work = p && ps != 0 && (ps >> 1) > c->attempted && (async || c->attempted == 0);
+        }
+        if (!work) {
+            // short spin (notification latency), then sleep on the futex
+            const int64_t t0 = now_ns();
+            bool got = false;
+            while (now_ns() - t0 < 50000) {
+                if (ctrl->pub_seq.load() != seq || c->stop.load()) {
+                    got = true;
+                    break;
+                }
+                cpu_relax();
+            }
+            if (!got) futex_wait(&ctrl->pub_seq, seq, 2000);
+            continue;
+        }
+        std::unique_lock<std::mutex> lk(c->install_mu);
+        uint64_t v;
+        int b;
+        if (!pin_latest(ctrl, r, &v, &b)) continue;
+        if (v <= c->attempted) {
+            r->pin.store(0);
+            continue;
+        }
+        if (c->attempted && v > c->attempted + 1) {
+            std::lock_guard<std::mutex> sl(c->stats_mu);
+            c->stats.skipped += v - c->attempted - 1;  // latest-wins
+        }
+        c->attempted = v;
+        const int64_t tp = ctrl->pub_time_ns.load();
+        const int64_t t0 = now_ns();
+        viper_model *p = c->chan ? c->chan->producer : nullptr;
+        viper_status st = p ? enqueue_install(c, p, v, b, c->ustream, true)
+                            : set_error(VIPER_E_STATE, "producer gone");
+        if (st == VIPER_OK) {
+            cudaError_t e = cudaStreamSynchronize(c->ustream);
+            if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
+        }
+        if (st == VIPER_OK) st = finish_install(c, v, (now_ns() - t0) / 1e3);
+        else {
+            r->status.store(st);
+            finish_install(c, v, (now_ns() - t0) / 1e3);
+        }
+        {
+            std::lock_guard<std::mutex> sl(c->stats_mu);
+            c->stats.t_notify_us = tp ? (t0 - tp) / 1e3 : 0.0;
+        }
+        lk.unlock();
+        fire_callback(c, v, st);
+    }
+}
+
+// ------------------------------------------------------------------ producer
+static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st) {
+    const int64_t t0 = now_ns();
+    if (v == 0 || v <= p->last_version)
+        return set_error(VIPER_E_VERSION, "publish(%llu) after %llu: versions strictly increase from 1",
+                         (unsigned long long)v, (unsigned long long)p->last_version);
+    Ctrl *ctrl = p->ctrl;
+    const int b = p->cur_snap ^ 1;
+    const uint64_t old_v = p->snap_version[b];
+    // Slot b still holds old_v: wait until no consumer reads it (latest-only
+    // buffer).  pub_state already names a newer version, so late
+    // pinners of old_v fail their re-validation.
+    if (old_v) {
+        const int nc = ctrl->ncons.load();
+        for (int i = 0; i < nc; i++) {
+            const int64_t w0 = now_ns();
+            while (ctrl->cons[i].active.load() && ctrl->cons[i].pin.load() == old_v) {
+                if (now_ns() - w0 > 10ll * 1000000000ll)
+                    return set_error(VIPER_E_TIMEOUT, "consumer %d kept snapshot v%llu pinned", i,
+                                     (unsigned long long)old_v);
+                cpu_relax();
+            }
+        }
+        // the DRAM-tier D2H of old_v must be finished before overwriting
+        if (p->cfg.tier == VIPER_TIER_DRAM) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
+    }
+    PackArgs a{};
+    a.items = p->man.d_items;
+    a.nitems = (uint32_t)p->man.items.size();
+    a.nchunks = p->man.nchunks;
+    a.src = p->d_src;
+    a.packed = p->d_snap[b];
+    a.seals = p->d_seal[b];
+    a.s = p->scratch;
+    a.version = v;
+    const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
+    if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
+    CUDA_TRY(launch_pack(a, p->geo, st));
+    if (timing) {
+        CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
+        p->timing_pending = true;
+    }
+    if (p->cfg.tier == VIPER_TIER_DRAM) {
+        // snapshot -> pinned host, on a side stream so the
+        // caller's stream is blocked only by the pack
+        CUDA_TRY(cudaEventRecord(p->ev_packed, st));
+        CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
+        CUDA_TRY(cudaMemcpyAsync(p->h_stage[b], p->d_snap[b], p->man.s_packed, cudaMemcpyDeviceToHost, p->side));
+        CUDA_TRY(cudaMemcpyAsync(p->h_seal[b], p->d_seal[b], sizeof(Seal) * p->man.nchunks,
+                                 cudaMemcpyDeviceToHost, p->side));
+        CUDA_TRY(cudaEventRecord(p->ev_ready[b], p->side));
+    } else {
+        CUDA_TRY(cudaEventRecord(p->ev_ready[b], st));
+    }
+    p->snap_version[b] = v;
+    p->cur_snap = b;
+    p->last_version = v;
+    ctrl->pub_state.store((v << 1) | (uint64_t)b);
+    ctrl->pub_time_ns.store(now_ns());
+
+    viper_status result = VIPER_OK;
+    if (p->cfg.mode == VIPER_SYNC) {
+        // SYNC: deliver + install inline, stream-ordered after the
+        // pack; return once every consumer swapped (or failed).
+        std::vector<viper_model *> cons;
+        {
+            std::lock_guard<std::mutex> lk(g_reg_mu);
+            cons = p->chan->consumers;
+        }
+        std::vector<std::unique_lock<std::mutex>> locks;
+        std::vector<viper_model *> launched;
+        for (viper_model *c : cons) {
+            std::unique_lock<std::mutex> lk(c->install_mu);
+            if (c->attempted >= v) continue;  // its update thread already did v
+            uint64_t pv;
+            int pb;
+            if (!pin_latest(ctrl, c->rec, &pv, &pb) || pv != v) continue;
+            c->attempted = v;
+            viper_status s = enqueue_install(c, p, v, b, st, p->cfg.tier == VIPER_TIER_DRAM);
+            if (s != VIPER_OK) {
+                c->rec->pin.store(0);
+                result = s;
+                continue;
+            }
+            launched.push_back(c);
+            locks.push_back(std::move(lk));
+        }
+        const int64_t ti = now_ns();
+        CUDA_TRY(cudaStreamSynchronize(st));
+        for (viper_model *c : launched) {
+            viper_status s = finish_install(c, v, (now_ns() - ti) / 1e3);
+            if (s != VIPER_OK && result == VIPER_OK) result = s;
+        }
+        locks.clear();
+        for (viper_model *c : launched) fire_callback(c, v, c->rec->last_status.load());
+    } else {
+        ctrl->pub_seq.fetch_add(1);
+        futex_wake_all(&ctrl->pub_seq);
+    }
+    {
+        std::lock_guard<std::mutex> lk(p->stats_mu);
+        p->stats.version = v;
+        p->stats.t_publish_us = (now_ns() - t0) / 1e3;
+        p->stats.last_status = result;
+    }
+    return result;
+}
+
+// -------------------------------------------------------------- registration
+static viper_status check_tensors(const viper_tensor *t, int32_t n) {
+    if (n < 0 || (n > 0 && !t)) return set_error(VIPER_E_INVAL, "bad tensor list");
+    for (int32_t i = 0; i < n; i++) {
+        if (t[i].nbytes && !t[i].dev_ptr) return set_error(VIPER_E_INVAL, "tensor %d: null dev_ptr", i);
+        if (t[i].dtype < VIPER_F32 || t[i].dtype > VIPER_BYTES) return set_error(VIPER_E_INVAL, "tensor %d: dtype", i);
+        if (t[i].nbytes > 0xFFFFFFFFull * 64) return set_error(VIPER_E_INVAL, "tensor %d too large", i);
+    }
+    return VIPER_OK;
+}
+
+static viper_status upload_ptrs(const std::vector<void *> &ptrs, void ***d_out) {
+    const size_t bytes = std::max<size_t>(ptrs.size(), 1) * sizeof(void *);
+    CUDA_TRY(cudaMalloc((void **)d_out, bytes));
+    if (!ptrs.empty()) CUDA_TRY(cudaMemcpy(*d_out, ptrs.data(), ptrs.size() * sizeof(void *), cudaMemcpyHostToDevice));
+    return VIPER_OK;
+}
+
+static void free_model(viper_model *m) {
+    if (!m) return;
+    if (m->upd.joinable()) {
+        m->stop.store(true);
+        if (m->ctrl) {
+            m->ctrl->pub_seq.fetch_add(1);
+            futex_wake_all(&m->ctrl->pub_seq);
+        }
+        m->upd.join();
+    }
+    cudaSetDevice(m->device);
+    cudaDeviceSynchronize();
+    if (m->rec) m->rec->active.store(0);
+    if (m->chan) {
+        {
+            std::lock_guard<std::mutex> lk(g_reg_mu);
+            auto &v = m->chan->consumers;
+            v.erase(std::remove(v.begin(), v.end(), m), v.end());
+            if (m->chan->producer == m) m->chan->producer = nullptr;
+        }
+        channel_close(m->chan);
+    }
+    cudaFree(m->man.d_items);
+    cudaFree(m->scratch_alloc);
+    cudaFree((void *)m->d_src);
+    cudaFree(m->snap_alloc);
+    cudaFree(m->d_slot[0]);
+    cudaFree(m->d_slot[1]);
+    cudaFree(m->slot1_alloc);
+    cudaFree(m->stage_alloc);
+    if (m->h_stage_alloc) cudaFreeHost(m->h_stage_alloc);
+    for (auto &e : m->ev_ready)
+        if (e) cudaEventDestroy(e);
+    for (auto &e : m->ev_t)
+        if (e) cudaEventDestroy(e);
+    if (m->ev_packed) cudaEventDestroy(m->ev_packed);
+    if (m->side) cudaStreamDestroy(m->side);
+    if (m->ustream) cudaStreamDestroy(m->ustream);
+    delete m;
+}
+
+static viper_status register_local(viper_model *m, const viper_tensor *tensors) {
+    viper_status st = channel_open(m->name, m->man, &m->chan);
+    if (st) return st;
+    m->ctrl = m->chan->ctrl;
+    m->ctrl_dev = m->chan->ctrl_dev;
+    const uint64_t S = m->man.s_packed;
+    const size_t seal_bytes = sizeof(Seal) * std::max<uint32_t>(m->man.nchunks, 1);
+    if (m->role == VIPER_PRODUCER) {
+        {
+            std::lock_guard<std::mutex> lk(g_reg_mu);
+            if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
+            m->chan->producer = m;
+        }
+        for (int32_t i = 0; i < m->man.n; i++) m->src_ptrs.push_back(tensors[i].dev_ptr);
+        if ((st = upload_ptrs(m->src_ptrs, (void ***)&m->d_src))) return st;
+        // two snapshot slots (latest + one being filled) + their seals
+        const uint64_t S_al = (S + 255) / 256 * 256;
+        const size_t bytes = 2 * S_al + 2 * seal_bytes;
+        CUDA_TRY(cudaMalloc(&m->snap_alloc, bytes));
+        CUDA_TRY(cudaMemset(m->snap_alloc, 0, bytes));  // padding bytes stay 0 forever
+        m->d_snap[0] = (uint8_t *)m->snap_alloc;
+        m->d_snap[1] = m->d_snap[0] + S_al;
+        m->d_seal[0] = (Seal *)(m->d_snap[1] + S_al);
+        m->d_seal[1] = (Seal *)((uint8_t *)m->d_seal[0] + seal_bytes);
+        for (auto &e : m->ev_ready) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
+        CUDA_TRY(cudaEventCreateWithFlags(&m->ev_packed, cudaEventDisableTiming));
+        if (m->cfg.tier == VIPER_TIER_DRAM) {
+            CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
+            CUDA_TRY(cudaHostAlloc(&m->h_stage_alloc, 2 * S_al + 2 * seal_bytes, cudaHostAllocPortable));
+            m->h_stage[0] = (uint8_t *)m->h_stage_alloc;
+            m->h_stage[1] = m->h_stage[0] + S_al;
+            m->h_seal[0] = (Seal *)(m->h_stage[1] + S_al);
+            m->h_seal[1] = (Seal *)((uint8_t *)m->h_seal[0] + seal_bytes);
+        }
+        return VIPER_OK;
+    }
+    // consumer
+    {
+        std::lock_guard<std::mutex> lk(g_reg_mu);
+        const int idx = m->ctrl->ncons.load();
+        if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+        m->cidx = idx;
+        m->rec = &m->ctrl->cons[idx];
+        m->rec_dev = &m->ctrl_dev->cons[idx];
+        m->rec->active.store(1);
+        m->ctrl->ncons.store(idx + 1);
+        m->chan->consumers.push_back(m);
+    }
+    for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[0].push_back(tensors[i].dev_ptr);
+    if (m->cfg.slot1) {
+        for (int32_t i = 0; i < m->man.n; i++) {
+            if (m->cfg.slot1[i].nbytes != m->man.nbytes[i] || (m->man.nbytes[i] && !m->cfg.slot1[i].dev_ptr))
+                return set_error(VIPER_E_INVAL, "slot1 tensor %d does not match", i);
+            m->slot_ptrs[1].push_back(m->cfg.slot1[i].dev_ptr);
+        }
+    } else {
+        CUDA_TRY(cudaMalloc(&m->slot1_alloc, std::max<uint64_t>(S, 256)));
+        for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[1].push_back((uint8_t *)m->slot1_alloc + m->man.offsets[i]);
+    }
+    for (int s = 0; s < 2; s++)
+        if ((st = upload_ptrs(m->slot_ptrs[s], (void ***)&m->d_slot[s]))) return st;
+    if (m->cfg.tier == VIPER_TIER_DRAM) {
+        CUDA_TRY(cudaMalloc(&m->stage_alloc, (S + 255) / 256 * 256 + seal_bytes));
+        m->d_stage = (uint8_t *)m->stage_alloc;
+        m->d_stage_seals = (Seal *)(m->d_stage + (S + 255) / 256 * 256);
+    }
+    CUDA_TRY(cudaStreamCreateWithFlags(&m->ustream, cudaStreamNonBlocking));
+    for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
+    m->upd = std::thread(update_loop, m);
+    return VIPER_OK;
+}
+
+}  // namespace vp
+
+using namespace vp;
+
+// =================================================================== C-ABI
+extern "C" {
+
+viper_status viper_xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
+viper_status viper_xproc_publish(viper_model *m, uint64_t version, cudaStream_t st);
+
+viper_status viper_register_model(const char *model_name, int32_t role, const viper_tensor *tensors, int32_t n,
+                                  const viper_config *cfg, const viper_bootstrap *bs, viper_model **out) {
+    try {
+        if (!out) return set_error(VIPER_E_INVAL, "out is NULL");
+        *out = nullptr;
+        if (!model_name || !*model_name) return set_error(VIPER_E_INVAL, "empty model name");
+        if (role != VIPER_PRODUCER && role != VIPER_CONSUMER) return set_error(VIPER_E_INVAL, "bad role %d", role);
+        viper_status st = check_tensors(tensors, n);
+        if (st) return st;
+        viper_config c{};
+        if (cfg) c = *cfg;
+        if (c.chunk_bytes == 0) c.chunk_bytes = 2ull << 20;
+        if (c.align == 0) c.align = 256;
+        if (c.align < 16 || (c.align & (c.align - 1))) return set_error(VIPER_E_INVAL, "align must be a power of 2 >= 16");
+        if (c.chunk_bytes % 256 || c.chunk_bytes % c.align) return set_error(VIPER_E_INVAL, "chunk_bytes must be a multiple of 256 and align");
+        if (c.tier != VIPER_TIER_GPU && c.tier != VIPER_TIER_DRAM) return set_error(VIPER_E_INVAL, "bad tier");
+        if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
+        if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER)
+            return set_error(VIPER_E_UNSUPPORTED, "fanout %d not supported", c.fanout);
+        int ndev = 0;
+        if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0)
+            return set_error(VIPER_E_CUDA, "no CUDA device (there is no CPU fallback)");
+        if (c.device < 0 || c.device >= ndev) return set_error(VIPER_E_INVAL, "bad device %d", c.device);
+        CUDA_TRY(cudaSetDevice(c.device));
+        viper_model *m = new viper_model();
+        m->name = model_name;
+        m->role = role;
+        m->device = c.device;
+        m->cfg = c;
+        st = build_manifest(m->man, tensors, n, c.chunk_bytes, c.align, c.device);
+        if (!st) st = alloc_scratch(m);
+        if (!st) {
+            m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device);
+            if (bs && bs->world > 1) {
+                m->xproc = true;
+                st = viper_xproc_register(m, tensors, bs);
+            } else {
+                st = register_local(m, tensors);
+            }
+        }
+        if (st) {
+            std::string keep = t_err;
+            free_model(m);
+            t_err = keep;
+            return st;
+        }
+        {
+            std::lock_guard<std::mutex> lk(m->stats_mu);
+            m->stats.s_packed = m->man.s_packed;
+            m->stats.nchunks = m->man.nchunks;
+            m->stats.nitems = m->man.items.size();
+        }
+        *out = m;
+        return VIPER_OK;
+    } catch (const std::exception &e) {
+        return set_error(VIPER_E_NOMEM, "register: %s", e.what());
+    }
+}
+
+viper_status viper_publish(viper_model *m, uint64_t version, void *cuda_stream) {
+    if (!m || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_PRODUCER) return set_error(VIPER_E_STATE, "publish on a consumer");
+    try {
+        if (cudaSetDevice(m->device) != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice");
+        if (m->xproc) return viper_xproc_publish(m, version, (cudaStream_t)cuda_stream);
+        return producer_publish(m, version, (cudaStream_t)cuda_stream);
+    } catch (const std::exception &e) {
+        return set_error(VIPER_E_NOMEM, "publish: %s", e.what());
+    }
+}
+
+viper_status viper_subscribe(viper_model *m, void (*on_update)(uint64_t, viper_status, void *), void *user) {
+    if (!m || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "subscribe on a producer");
+    std::lock_guard<std::mutex> lk(m->cb_mu);
+    m->cb = on_update;
+    m->cb_user = user;
+    return VIPER_OK;
+}
+
+viper_status viper_acquire_latest(viper_model *m, uint64_t min_version, int64_t timeout_us, viper_view *out) {
+    if (!m || !out || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "acquire on a producer");
+    ConsRec *r = m->rec;
+    const int64_t deadline = timeout_us < 0 ? INT64_MAX : now_ns() + timeout_us * 1000;
+    for (;;) {
+        const uint32_t seq = r->done_seq.load();
+        const uint64_t s = r->state.load();
+        if (s == 0 || (s >> 1) < min_version) {
+            const int64_t now = now_ns();
+            if (timeout_us == 0) return set_error(VIPER_E_NOVERSION, "no version >= %llu installed",
+                                                  (unsigned long long)min_version);
+            if (now >= deadline) return set_error(VIPER_E_TIMEOUT, "acquire timed out");
+            const int64_t left_us = (deadline - now) / 1000;
+            futex_wait(&r->done_seq, seq, std::min<int64_t>(left_us, 1000));
+            continue;
+        }
+        const int slot = (int)(s & 1);
+        r->ref[slot].fetch_add(1);
+        if (r->state.load() == s) {
+            std::lock_guard<std::mutex> lk(m->views_mu);
+            const uint64_t t = m->next_ticket++;
+            m->views[t] = ViewTicket{slot};
+            out->version = s >> 1;
+            out->slot = slot;
+            out->ntensors = m->man.n;
+            out->dev_ptrs = m->slot_ptrs[slot].data();
+            out->ticket = t;
+            return VIPER_OK;
+        }
+        r->ref[slot].fetch_sub(1);  // swapped under us: retry
+    }
+}
+
+struct ReleaseCtx {
+    ConsRec *r;
+    int slot;
+};
+
+static void CUDART_CB release_host_fn(void *p) {
+    ReleaseCtx *c = (ReleaseCtx *)p;
+    c->r->ref[c->slot].fetch_sub(1);
+    delete c;
+}
+
+viper_status viper_release(viper_model *m, const viper_view *view, void *cuda_stream) {
+    if (!m || !view || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "release on a producer");
+    int slot;
+    {
+        std::lock_guard<std::mutex> lk(m->views_mu);
+        auto it = m->views.find(view->ticket);
+        if (it == m->views.end() || it->second.slot != view->slot)
+            return set_error(VIPER_E_STATE, "unknown or already released view (ticket %llu)",
+                             (unsigned long long)view->ticket);
+        slot = it->second.slot;
+        m->views.erase(it);
+    }
+    if (cuda_stream) {
+        cudaSetDevice(m->device);
+        ReleaseCtx *c = new ReleaseCtx{m->rec, slot};
+        cudaError_t e = cudaLaunchHostFunc((cudaStream_t)cuda_stream, release_host_fn, c);
+        if (e != cudaSuccess) {
+            delete c;
+            m->rec->ref[slot].fetch_sub(1);
+            return set_error(VIPER_E_CUDA, "cudaLaunchHostFunc: %s", cudaGetErrorString(e));
+        }
+        return VIPER_OK;
+    }
+    m->rec->ref[slot].fetch_sub(1);
+    return VIPER_OK;
+}
+
+viper_status viper_wait_installed(viper_model *m, uint64_t v, int64_t timeout_us) {
+    if (!m || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "wait_installed on a producer");
+    ConsRec *r = m->rec;
+    const int64_t deadline = timeout_us < 0 ? INT64_MAX : now_ns() + timeout_us * 1000;
+    for (;;) {
+        const uint32_t seq = r->done_seq.load();
+        if ((r->state.load() >> 1) >= v) return VIPER_OK;
+        if (r->done_version.load() >= v && r->last_status.load() != VIPER_OK) return r->last_status.load();
+        const int64_t now = now_ns();
+        if (now >= deadline) return set_error(VIPER_E_TIMEOUT, "version %llu not installed in time", (unsigned long long)v);
+        futex_wait(&r->done_seq, seq, std::min<int64_t>((deadline - now) / 1000, 1000));
+    }
+}
+
+viper_status viper_get_stats(viper_model *m, viper_stats *out) {
+    if (!m || !out) return set_error(VIPER_E_INVAL, "null");
+    if (m->role == VIPER_PRODUCER && m->timing_pending && cudaEventQuery(m->ev_t[1]) == cudaSuccess) {
+        float ms = 0;
+        if (cudaEventElapsedTime(&ms, m->ev_t[0], m->ev_t[1]) == cudaSuccess) {
+            std::lock_guard<std::mutex> lk(m->stats_mu);
+            m->stats.t_pack_dev_us = ms * 1e3;
+        }
+        m->timing_pending = false;
+    }
+    std::lock_guard<std::mutex> lk(m->stats_mu);
+    *out = m->stats;
+    out->nconsumers = m->ctrl ? m->ctrl->ncons.load() : 0;
+    return VIPER_OK;
+}
+
+viper_status viper_layout(viper_model *m, uint64_t *s_packed, uint64_t *offsets, int32_t n) {
+    if (!m) return set_error(VIPER_E_INVAL, "null model");
+    if (s_packed) *s_packed = m->man.s_packed;
+    if (offsets) {
+        if (n < m->man.n) return set_error(VIPER_E_INVAL, "offsets array too small");
+        for (int32_t i = 0; i < m->man.n; i++) offsets[i] = m->man.offsets[i];
+    }
+    return VIPER_OK;
+}
+
+viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_seals, uint64_t *nchunks) {
+    if (!m) return set_error(VIPER_E_INVAL, "null model");
+    if (nchunks) *nchunks = m->man.nchunks;
+    if (m->role == VIPER_PRODUCER) {
+        const int b = m->cur_snap;
+        if (dev_packed) *dev_packed = m->d_snap[b];
+        if (dev_seals) *dev_seals = m->d_seal[b];
+    } else {
+        if (dev_packed) *dev_packed = m->d_stage;
+        if (dev_seals) *dev_seals = m->d_stage_seals;
+    }
+    return VIPER_OK;
+}
+
+viper_status viper_debug_fault_next(viper_model *m) {
+    if (!m || m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "consumer only");
+    m->fault_next.store(true);
+    return VIPER_OK;
+}
+
+viper_status viper_unregister(viper_model *m) {
+    if (!m) return set_error(VIPER_E_INVAL, "null model");
+    if (m->closed.exchange(true)) return set_error(VIPER_E_STATE, "double unregister");
+    free_model(m);
+    return VIPER_OK;
+}
+
+const char *viper_strerror(viper_status st) {
+    switch (st) {
+        case VIPER_OK: return "VIPER_OK";
+        case VIPER_E_INVAL: return "VIPER_E_INVAL";
+        case VIPER_E_NOMEM: return "VIPER_E_NOMEM";
+        case VIPER_E_CUDA: return "VIPER_E_CUDA";
+        case VIPER_E_VERSION: return "VIPER_E_VERSION";
+        case VIPER_E_CHECKSUM: return "VIPER_E_CHECKSUM";
+        case VIPER_E_TIMEOUT: return "VIPER_E_TIMEOUT";
+        case VIPER_E_NOVERSION: return "VIPER_E_NOVERSION";
+        case VIPER_E_STATE: return "VIPER_E_STATE";
+        case VIPER_E_UNSUPPORTED: return "VIPER_E_UNSUPPORTED";
+        case VIPER_E_PEER: return "VIPER_E_PEER";
+        default: return "VIPER_E_UNKNOWN";
+    }
+}
+
+const char *viper_last_error(void) { return t_err.c_str(); }
+const char *viper_version(void) { return "viper-b200 0.1 (sm_100a)"; }
+
+}  // extern "C"

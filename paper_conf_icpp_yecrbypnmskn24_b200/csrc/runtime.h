@@ -1,0 +1,148 @@
+// runtime.h -- host-side engine state of libviper.so (internal).
+//
+// Control plane: a Ctrl block in pinned, device-mapped
+// host memory (in-process channel) or in a POSIX shared-memory segment
+// registered with CUDA (cross-process channel) holds
+//   pub_state  = (version << 1) | snapshot_slot   -- what the producer published
+//   per consumer: state = (version << 1) | slot    -- what it serves (flipped by
+//                 the install kernel from the device), pin (snapshot version it
+//                 is reading), ref[2] (readers per slot), done_version/done_seq.
+// All host-side accesses are seq_cst std::atomic; the device writes state,
+// pin and status with system-scope fenced stores (kernels.cu finalize_install).
+#pragma once
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <map>
+#include <mutex>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "../../include/viper.h"
+#include "vp_internal.h"
+
+namespace vp {
+
+constexpr int kMaxConsumers = 16;
+constexpr uint64_t kCtrlMagic = 0x5649504552435431ull;  // "VIPERCT1"
+
+struct alignas(64) ConsRec {
+    std::atomic<uint64_t> state;         // (v << 1) | slot, 0 = nothing installed (device-written)
+    std::atomic<uint64_t> pin;           // snapshot version being read, 0 = none (device-cleared)
+    std::atomic<int32_t> status;         // result of the last install kernel (device-written)
+    std::atomic<int32_t> active;
+    std::atomic<int64_t> ref[2];         // readers pinning each slot
+    std::atomic<uint64_t> done_version;  // last version processed (installed or failed)
+    std::atomic<uint32_t> done_seq;      // futex word, bumped after each install attempt
+    std::atomic<int32_t> last_status;
+    std::atomic<uint64_t> p1_done;       // scatter-allgather: phase-1 version finished
+    std::atomic<uint64_t> p2_done;       // scatter-allgather: phase-2 version finished
+};
+
+struct alignas(64) Ctrl {
+    uint64_t magic;
+    std::atomic<uint64_t> pub_state;     // (v << 1) | snapshot slot, 0 = none
+    std::atomic<uint32_t> pub_seq;       // futex word, bumped on each publish
+    std::atomic<uint32_t> closing;
+    std::atomic<int64_t> pub_time_ns;    // CLOCK_MONOTONIC of the last publish notification
+    std::atomic<int32_t> ncons;
+    ConsRec cons[kMaxConsumers];
+};
+
+struct Manifest {
+    int32_t n = 0;
+    std::vector<uint64_t> nbytes, offsets;
+    uint64_t s_packed = 0, chunk_bytes = 0;
+    uint32_t align = 0;
+    std::vector<Item> items;
+    uint32_t nchunks = 0;
+    Item *d_items = nullptr;
+};
+
+struct Channel;
+
+struct ViewTicket {
+    int32_t slot;
+};
+
+}  // namespace vp
+
+struct viper_model {
+    std::string name;
+    int32_t role = 0, device = 0;
+    viper_config cfg{};
+    vp::Manifest man;
+    vp::Geometry geo{};
+    vp::Scratch scratch{};
+    void *scratch_alloc = nullptr;
+    vp::Channel *chan = nullptr;       // in-process channel (registry entry)
+    vp::Ctrl *ctrl = nullptr;          // host view of the control block
+    vp::Ctrl *ctrl_dev = nullptr;      // device view (mapped)
+    bool xproc = false;
+    std::atomic<bool> closed{false};
+
+    // ---------------- producer
+    std::vector<void *> src_ptrs;
+    const uint8_t **d_src = nullptr;
+    uint8_t *d_snap[2] = {nullptr, nullptr};
+    vp::Seal *d_seal[2] = {nullptr, nullptr};
+    void *snap_alloc = nullptr;
+    cudaEvent_t ev_ready[2] = {nullptr, nullptr};   // snapshot slot b complete
+    cudaEvent_t ev_packed = nullptr;
+    cudaEvent_t ev_t[2] = {nullptr, nullptr};        // VIPER_FLAG_TIMING: around the kernel
+    bool timing_pending = false;
+    cudaStream_t side = nullptr;                     // DRAM-tier D2H stream
+    uint8_t *h_stage[2] = {nullptr, nullptr};        // DRAM tier (pinned)
+    vp::Seal *h_seal[2] = {nullptr, nullptr};
+    void *h_stage_alloc = nullptr;
+    uint64_t snap_version[2] = {0, 0};
+    uint64_t last_version = 0;
+    int cur_snap = 1;
+
+    // ---------------- consumer
+    int32_t cidx = -1;
+    vp::ConsRec *rec = nullptr, *rec_dev = nullptr;
+    std::vector<void *> slot_ptrs[2];
+    uint8_t **d_slot[2] = {nullptr, nullptr};
+    void *slot1_alloc = nullptr;
+    uint8_t *d_stage = nullptr;                      // DRAM tier device staging
+    vp::Seal *d_stage_seals = nullptr;
+    void *stage_alloc = nullptr;
+    cudaStream_t ustream = nullptr;
+    std::thread upd;
+    std::atomic<bool> stop{false};
+    std::mutex install_mu;
+    uint64_t attempted = 0;
+    std::atomic<bool> fault_next{false};
+    std::mutex cb_mu;
+    void (*cb)(uint64_t, viper_status, void *) = nullptr;
+    void *cb_user = nullptr;
+    std::mutex views_mu;
+    std::unordered_map<uint64_t, vp::ViewTicket> views;
+    uint64_t next_ticket = 1;
+
+    // ---------------- stats
+    std::mutex stats_mu;
+    viper_stats stats{};
+};
+
+namespace vp {
+
+struct Channel {
+    std::string name;
+    Ctrl *ctrl = nullptr, *ctrl_dev = nullptr;
+    viper_model *producer = nullptr;
+    std::vector<viper_model *> consumers;
+    int refs = 0;
+    std::vector<uint64_t> nbytes;  // manifest check
+};
+
+// runtime.cpp helpers used by other translation units
+viper_status set_error(viper_status st, const char *fmt, ...);
+int64_t now_ns();
+void futex_wake_all(std::atomic<uint32_t> *w);
+void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us);
+
+}  // namespace vp

@@ -1,0 +1,52 @@
+"""GPU side of the input generator: ctypes wrapper of synth/libvgen.so (harness
+kernel writing VGEN bits into producer tensors; see synth/__init__.py)."""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+_LIB = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libvgen.so")
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_LIB):
+            raise ImportError(f"{_LIB} missing -- run __graft_entry__.build()")
+        _lib = C.CDLL(_LIB)
+        _lib.vgen_fill.argtypes = [C.c_void_p, C.c_uint64, C.c_uint64, C.c_uint64, C.c_int32, C.c_uint64, C.c_void_p]
+        _lib.vgen_fill.restype = C.c_int
+        _lib.l2_flush.argtypes = [C.c_void_p, C.c_uint64, C.c_void_p]
+        _lib.l2_flush.restype = C.c_int
+    return _lib
+
+
+def _sp(stream):
+    return None if stream is None else C.c_void_p(stream.cuda_stream)
+
+
+def fill(t, seed: int, version: int, index: int, dtype: int, stream=None):
+    """Write VGEN(seed, version, index, e) into CUDA tensor t (raw bytes)."""
+    from . import DTYPE_SIZE
+    n = t.numel() * t.element_size() // DTYPE_SIZE[dtype]
+    if lib().vgen_fill(C.c_void_p(t.data_ptr()), seed, version, index, dtype, n, _sp(stream)) != 0:
+        raise RuntimeError("vgen_fill failed")
+
+
+def fill_model(tensors, specs, seed: int, version: int, stream=None):
+    for i, (t, s) in enumerate(zip(tensors, specs)):
+        fill(t, seed, version, i, s[1], stream)
+
+
+def alloc_model(specs, device="cuda:0"):
+    """Allocate one CUDA tensor per spec (torch dtype matching the spec)."""
+    import torch
+    from . import F32, BF16, F16
+    dt = {F32: torch.float32, BF16: torch.bfloat16, F16: torch.float16}
+    return [torch.empty(s[2], dtype=dt.get(s[1], torch.uint8), device=device) for s in specs]
+
+
+def l2_flush(buf, stream=None):
+    if lib().l2_flush(C.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(), _sp(stream)) != 0:
+        raise RuntimeError("l2_flush failed")

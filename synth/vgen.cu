@@ -1,0 +1,66 @@
+// vgen.cu -- harness kernel (NOT part of the method): writes VGEN(seed, v, t, e)
+// into a producer tensor on the GPU, standing in for the training step's
+// optimizer write between model versions.  Same counter-based generator as
+// synth.vgen_numpy (see synth/__init__.py for the definition); no state is
+// shared with the CPU side, both compute it from (seed, v, t, e).
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace {
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+uint64_t splitmix64_host(uint64_t x) {
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+template <int DT>
+__global__ void vgen_kernel(uint8_t *out, uint64_t key, uint64_t nelem) {
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < nelem; e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t h = splitmix64(key + e);
+        const uint64_t sign = h >> 63, ex = (h >> 32) & 3;
+        if (DT == 0) {
+            reinterpret_cast<uint32_t *>(out)[e] = (uint32_t)((sign << 31) | ((119 + ex) << 23) | (h & 0x7FFFFF));
+        } else if (DT == 1) {
+            reinterpret_cast<uint16_t *>(out)[e] = (uint16_t)((sign << 15) | ((119 + ex) << 7) | (h & 0x7F));
+        } else if (DT == 2) {
+            reinterpret_cast<uint16_t *>(out)[e] = (uint16_t)((sign << 15) | ((7 + ex) << 10) | (h & 0x3FF));
+        } else {
+            out[e] = (uint8_t)(h & 0xFF);
+        }
+    }
+}
+
+}  // namespace
+
+extern "C" int vgen_fill(void *dev_ptr, uint64_t seed, uint64_t version, uint64_t t, int32_t dtype, uint64_t nelem,
+                         void *stream) {
+    if (nelem == 0) return 0;
+    const uint64_t key = splitmix64_host(seed ^ splitmix64_host((version << 20) ^ t));
+    const int block = 256;
+    uint64_t want = (nelem + block - 1) / block;
+    const int grid = (int)(want > 148 * 16 ? 148 * 16 : want);
+    cudaStream_t st = (cudaStream_t)stream;
+    uint8_t *p = (uint8_t *)dev_ptr;
+    switch (dtype) {
+        case 0: vgen_kernel<0><<<grid, block, 0, st>>>(p, key, nelem); break;
+        case 1: vgen_kernel<1><<<grid, block, 0, st>>>(p, key, nelem); break;
+        case 2: vgen_kernel<2><<<grid, block, 0, st>>>(p, key, nelem); break;
+        case 3: vgen_kernel<3><<<grid, block, 0, st>>>(p, key, nelem); break;
+        default: return -1;
+    }
+    return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+
+// Flush L2 between timed steps: write `bytes` (> L2) of scratch.
+extern "C" int l2_flush(void *dev_ptr, uint64_t bytes, void *stream) {
+    return cudaMemsetAsync(dev_ptr, (int)(bytes & 0xFF), bytes, (cudaStream_t)stream) == cudaSuccess ? 0 : -3;
+}

@@ -1,0 +1,382 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the oracle, element by
+element on the same seeded VGEN inputs, plus the protocol invariants
+ on the device path.  Bit-exact throughout: this is
+byte work."""
+import threading
+import time
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import transfer as T
+from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+from synth import gpu as G
+
+pytestmark = pytest.mark.gpu
+_uid = [0]
+
+
+def uname(p="m"):
+    _uid[0] += 1
+    return f"{p}-{_uid[0]}-{time.monotonic_ns()}"
+
+
+def host_bytes(t):
+    return t.detach().contiguous().view(torch.uint8).reshape(-1).cpu().numpy() if t.numel() else np.zeros(0, np.uint8)
+
+
+def expect(specs, seed, v):
+    return [synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
+
+
+def oracle_packed_and_seals(specs, seed, v, chunk_bytes, align=256):
+    ts = expect(specs, seed, v)
+    off, s = T.layout([t.size for t in ts], align)
+    p = T.pack(ts, off, s)
+    return p, T.seal(p, chunk_bytes, v), off
+
+
+def _raw_u64(ptr, count):
+    """`count` uint64 words at device pointer ptr (as an int64 tensor)."""
+    like = torch.empty(2 * max(count, 1), dtype=torch.int32, device="cuda")
+    return V._from_ptr(ptr, like).view(torch.int64)[:count]
+
+
+def device_packed_and_seals(prod):
+    p, s, n = prod.debug_buffers()
+    S, _ = prod.layout()
+    torch.cuda.synchronize()
+    packed = V._from_ptr(p, torch.empty(S, dtype=torch.uint8, device="cuda")) if S else torch.empty(0, dtype=torch.uint8)
+    seals = _raw_u64(s, 2 * n)
+    return host_bytes(packed), seals.cpu().numpy().view(np.uint64).reshape(n, 2)
+
+
+def check_slot(view, cons_like, specs, seed, v):
+    got = view.tensors(cons_like)
+    exp = expect(specs, seed, v)
+    for i, (g, e) in enumerate(zip(got, exp)):
+        assert np.array_equal(host_bytes(g), e), f"tensor {i} differs at version {v}"
+
+
+def make_pair(specs, seed, ncons=1, **kw):
+    prod_t = G.alloc_model(specs)
+    cons_t = [G.alloc_model(specs) for _ in range(ncons)]
+    name = uname()
+    ckw = {k: v for k, v in kw.items() if k in ("tier", "chunk_bytes", "align")}
+    cons = [V.Model(name, V.CONSUMER, ct, **ckw) for ct in cons_t]
+    prod = V.Model(name, V.PRODUCER, prod_t, **kw)
+    return prod, prod_t, cons, cons_t
+
+
+def close_all(prod, cons):
+    for c in cons:
+        c.close()
+    prod.close()
+
+
+# ------------------------------------------------------------------ C1 (BJ configs[0])
+@pytest.mark.parametrize("tier", [V.TIER_GPU, V.TIER_DRAM])
+@pytest.mark.parametrize("mode", [V.SYNC, V.ASYNC])
+def test_c1_ptychonn_10_versions(tier, mode):
+    specs = synth.model_specs("ptychonn")
+    seed = synth.SEEDS["ptychonn"]
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, tier=tier, mode=mode)
+    try:
+        for v in range(1, 11):
+            G.fill_model(prod_t, specs, seed, v)
+            prod.publish(v)
+            if mode == V.ASYNC:
+                cons[0].wait_installed(v)
+            # producer snapshot and seals == oracle pack/seal of the same version
+            if mode == V.SYNC or v == 10:
+                p_dev, s_dev = device_packed_and_seals(prod)
+                p_or, s_or, _ = oracle_packed_and_seals(specs, seed, v, 2 << 20)
+                assert np.array_equal(p_dev, p_or)
+                assert np.array_equal(s_dev, s_or)
+            view = cons[0].acquire_latest(min_version=v, timeout_us=5_000_000)
+            assert view.version == v
+            check_slot(view, cons_t[0], specs, seed, v)
+            cons[0].release(view)
+        st = cons[0].stats()
+        assert st["installs"] >= 1 and st["failures"] == 0
+    finally:
+        close_all(prod, cons)
+
+
+# ----------------------------------------------------- ragged lists, several consumers
+@pytest.mark.parametrize("seed", range(6))
+def test_ragged_tensor_lists_many_chunks(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 40))
+    specs = []
+    for i in range(n):
+        dt = int(rng.choice([synth.F32, synth.BF16, synth.F16, synth.BYTES]))
+        ne = int(rng.choice([0, 1, 3, 7, 255, 1023, int(rng.integers(1, 70000))]))
+        specs.append((f"t{i}", dt, (ne,)))
+    chunk = int(rng.choice([256, 4096, 65536]))
+    align = int(rng.choice([16, 256]))
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=3, chunk_bytes=chunk, align=align)
+    try:
+        for v in (1, 2, 5):
+            G.fill_model(prod_t, specs, 77 + seed, v)
+            prod.publish(v)
+            p_dev, s_dev = device_packed_and_seals(prod)
+            p_or, s_or, _ = oracle_packed_and_seals(specs, 77 + seed, v, chunk, align)
+            assert np.array_equal(p_dev, p_or)
+            assert np.array_equal(s_dev, s_or)
+            for c, ct in zip(cons, cons_t):
+                view = c.acquire_latest()
+                assert view.version == v
+                check_slot(view, ct, specs, 77 + seed, v)
+                c.release(view)
+    finally:
+        close_all(prod, cons)
+
+
+def test_unaligned_tensor_pointers():
+    """Tensors that are byte-offset views (not 16-B aligned) take the word path."""
+    specs = [("a", synth.BYTES, (1001,)), ("b", synth.BYTES, (4099,)), ("c", synth.BYTES, (37,))]
+    base_p = torch.empty(6000, dtype=torch.uint8, device="cuda")
+    base_c = torch.empty(6000, dtype=torch.uint8, device="cuda")
+    prod_t = [base_p[1:1002], base_p[1003:5102], base_p[5103:5140]]
+    cons_t = [base_c[3:1004], base_c[1005:5104], base_c[5105:5142]]
+    name = uname()
+    cons = V.Model(name, V.CONSUMER, cons_t, chunk_bytes=1024)
+    prod = V.Model(name, V.PRODUCER, prod_t, chunk_bytes=1024)
+    try:
+        for v in (1, 2, 3):
+            G.fill_model(prod_t, specs, 5, v)
+            prod.publish(v)
+            p_dev, s_dev = device_packed_and_seals(prod)
+            p_or, s_or, _ = oracle_packed_and_seals(specs, 5, v, 1024)
+            assert np.array_equal(p_dev, p_or) and np.array_equal(s_dev, s_or)
+            view = cons.acquire_latest()
+            # slot 0 is the unaligned caller view, slot 1 the library copy
+            check_slot(view, cons_t, specs, 5, v)
+            cons.release(view)
+    finally:
+        close_all(prod, [cons])
+
+
+def test_empty_model():
+    name = uname()
+    cons = V.Model(name, V.CONSUMER, [], device=0)
+    prod = V.Model(name, V.PRODUCER, [], device=0)
+    try:
+        prod.publish(1)
+        view = cons.acquire_latest()
+        assert view.version == 1 and view.ptrs == []
+        cons.release(view)
+    finally:
+        close_all(prod, [cons])
+
+
+# ---------------------------------------------------------------- protocol on device
+def test_fault_injection_keeps_old_version():
+    specs = synth.model_specs("ptychonn")
+    seed = 11
+    prod, prod_t, cons, cons_t = make_pair(specs, seed)
+    try:
+        G.fill_model(prod_t, specs, seed, 1)
+        prod.publish(1)
+        cons[0].fault_next()
+        G.fill_model(prod_t, specs, seed, 2)
+        with pytest.raises(V.ViperError) as ei:
+            prod.publish(2)
+        assert ei.value.status == V.E_CHECKSUM
+        view = cons[0].acquire_latest()
+        assert view.version == 1
+        check_slot(view, cons_t[0], specs, seed, 1)
+        cons[0].release(view)
+        assert cons[0].stats()["failures"] == 1
+        G.fill_model(prod_t, specs, seed, 3)
+        prod.publish(3)
+        view = cons[0].acquire_latest()
+        assert view.version == 3
+        check_slot(view, cons_t[0], specs, seed, 3)
+        cons[0].release(view)
+    finally:
+        close_all(prod, cons)
+
+
+def test_version_and_view_errors():
+    specs = [("w", synth.F32, (1000,))]
+    prod, prod_t, cons, cons_t = make_pair(specs, 1)
+    try:
+        with pytest.raises(V.ViperError) as ei:
+            cons[0].acquire_latest(timeout_us=0)
+        assert ei.value.status == V.E_NOVERSION
+        with pytest.raises(V.ViperError) as ei:
+            prod.publish(0)
+        assert ei.value.status == V.E_VERSION
+        prod.publish(4)
+        for bad in (4, 3):
+            with pytest.raises(V.ViperError) as ei:
+                prod.publish(bad)
+            assert ei.value.status == V.E_VERSION
+        view = cons[0].acquire_latest()
+        cons[0].release(view)
+        with pytest.raises(V.ViperError) as ei:
+            cons[0].release(view)
+        assert ei.value.status == V.E_STATE
+        with pytest.raises(V.ViperError) as ei:
+            cons[0].publish(9)
+        assert ei.value.status == V.E_STATE
+        with pytest.raises(V.ViperError) as ei:
+            cons[0].acquire_latest(min_version=5, timeout_us=20_000)
+        assert ei.value.status == V.E_TIMEOUT
+    finally:
+        close_all(prod, cons)
+
+
+def test_writer_waits_for_pinned_slot():
+    """A reader pinning v keeps v's slot intact while v+1 and v+2 are published;
+    v+2 (which needs that slot) waits for the release (a7)."""
+    specs = [("w", synth.F32, (300_000,)), ("b", synth.F32, (77,))]
+    seed = 3
+    prod, prod_t, cons, cons_t = make_pair(specs, seed)
+    try:
+        G.fill_model(prod_t, specs, seed, 1)
+        prod.publish(1)
+        view = cons[0].acquire_latest()
+        G.fill_model(prod_t, specs, seed, 2)
+        prod.publish(2)                      # other slot: no wait
+        def late_release():
+            time.sleep(0.2)
+            check_slot(view, cons_t[0], specs, seed, 1)  # still v1 while pinned
+            cons[0].release(view)
+        th = threading.Thread(target=late_release)
+        th.start()
+        G.fill_model(prod_t, specs, seed, 3)
+        t0 = time.monotonic()
+        prod.publish(3)                      # needs view's slot
+        waited = time.monotonic() - t0
+        th.join()
+        assert waited > 0.15
+        assert cons[0].stats()["writer_wait_us"] > 1.5e5
+        v3 = cons[0].acquire_latest()
+        assert v3.version == 3
+        check_slot(v3, cons_t[0], specs, seed, 3)
+        cons[0].release(v3)
+    finally:
+        close_all(prod, cons)
+
+
+def test_stream_ordered_release():
+    specs = [("w", synth.F32, (4096,))]
+    prod, prod_t, cons, cons_t = make_pair(specs, 2)
+    try:
+        G.fill_model(prod_t, specs, 2, 1)
+        prod.publish(1)
+        s = torch.cuda.Stream()
+        view = cons[0].acquire_latest()
+        with torch.cuda.stream(s):
+            torch.cuda._sleep(20_000_000)  # ~10 ms of reader work on the slot's stream
+        cons[0].release(view, stream=s)
+        G.fill_model(prod_t, specs, 2, 2)
+        prod.publish(2)
+        G.fill_model(prod_t, specs, 2, 3)
+        prod.publish(3)  # waits until the stream passed the release
+        s.synchronize()
+        v = cons[0].acquire_latest()
+        assert v.version == 3
+        cons[0].release(v)
+    finally:
+        close_all(prod, cons)
+
+
+def test_no_torn_reads_under_async_publishes():
+    """Readers acquire -> compare every byte of the view with VGEN(view.version)
+    on the GPU -> release, while the producer publishes back to back (ASYNC)."""
+    specs = [(f"t{i}", synth.F32, (50_000 + 13 * i,)) for i in range(8)]
+    seed = 99
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.ASYNC)
+    stop = threading.Event()
+    errors, seen = [], []
+
+    def reader():
+        torch.cuda.set_device(0)
+        s = torch.cuda.Stream()
+        exp_t = G.alloc_model(specs)
+        last = 0
+        with torch.cuda.stream(s):
+            while not stop.is_set():
+                try:
+                    view = cons[0].acquire_latest(timeout_us=100_000)
+                except V.ViperError:
+                    continue
+                if view.version < last:
+                    errors.append(("regress", last, view.version))
+                last = view.version
+                G.fill_model(exp_t, specs, seed, view.version, stream=s)
+                got = view.tensors(cons_t[0])
+                bad = sum(int((g.view(torch.uint8) != e.view(torch.uint8)).sum()) for g, e in zip(got, exp_t))
+                if bad:
+                    errors.append(("torn", view.version, bad))
+                seen.append(view.version)
+                cons[0].release(view, stream=s)
+                s.synchronize()
+
+    ths = [threading.Thread(target=reader) for _ in range(2)]
+    try:
+        for th in ths:
+            th.start()
+        ps = torch.cuda.Stream()
+        for v in range(1, 301):
+            with torch.cuda.stream(ps):
+                G.fill_model(prod_t, specs, seed, v, stream=ps)
+                prod.publish(v, stream=ps)
+            if v % 50 == 0:
+                time.sleep(0.01)
+        cons[0].wait_installed(300)
+        time.sleep(0.05)
+        stop.set()
+        for th in ths:
+            th.join()
+        assert not errors, errors[:5]
+        assert len(seen) >= 20
+        assert cons[0].acquire_latest().version == 300
+    finally:
+        stop.set()
+        close_all(prod, cons)
+
+
+# ----------------------------------------------- BJ-sized models in 1-GPU loopback
+@pytest.mark.parametrize("name", ["resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
+def test_full_size_loopback_sampled(name):
+    """Full BASELINE.json model sizes, single-GPU loopback (the launch config
+    bench.py times): every seal's version; sampled chunk seals recomputed by the
+    oracle; sampled tensor byte ranges vs VGEN; all slot tensors == producer
+    tensors (replica identity at any size)."""
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.SYNC)
+    try:
+        for v in (1, 2):
+            G.fill_model(prod_t, specs, seed, v)
+            prod.publish(v)
+        torch.cuda.synchronize()
+        S, offsets = prod.layout()
+        p, sp, n = prod.debug_buffers()
+        seals = _raw_u64(sp, 2 * n).cpu().numpy().view(np.uint64).reshape(n, 2)
+        assert np.all(seals[:, 0] == 2)
+        rng = np.random.default_rng(0)
+        for c in sorted({0, n - 1, *rng.integers(0, n, 4).tolist()}):
+            assert int(seals[c, 1]) == T.expected_chunk_seal(specs, seed, 2, offsets, S, 2 << 20, c), c
+        view = cons[0].acquire_latest()
+        assert view.version == 2
+        got = view.tensors(cons_t[0])
+        for g, pt in zip(got, prod_t):
+            assert torch.equal(g.view(torch.uint8), pt.view(torch.uint8))
+        for i in sorted({0, len(specs) - 1, *rng.integers(0, len(specs), 6).tolist()}):
+            nb = synth.nbytes_of(specs[i])
+            lo = int(rng.integers(0, max(nb - 4096, 1)))
+            hi = min(nb, lo + 4096)
+            b = host_bytes(got[i].view(torch.uint8).reshape(-1)[lo:hi])
+            assert np.array_equal(b, synth.vgen_bytes_range(seed, 2, i, specs[i][1], lo, hi))
+        cons[0].release(view)
+    finally:
+        close_all(prod, cons)
+        torch.cuda.empty_cache()
