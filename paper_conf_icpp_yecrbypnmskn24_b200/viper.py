@@ -169,7 +169,7 @@ class _CAI:
         import torch
         typestr = {torch.float32: "<f4", torch.float16: "<f2", torch.uint8: "|u1", torch.int16: "<i2",
                    torch.int32: "<i4"}[t.dtype if t.dtype != torch.bfloat16 else torch.int16]
-        self.__cuda_array_interface__ = {"shape": tuple(t.shape), "typestr": typestr, "data": (ptr, True),
+        self.__cuda_array_interface__ = {"shape": tuple(t.shape), "typestr": typestr, "data": (ptr, False),
                                          "version": 3, "strides": None}
 
 
