@@ -95,9 +95,11 @@ enum { VIPER_SYNC = 0,   /* publish returns after every consumer installed v (or
                             delivery and install proceed in the background       */
 
 /* Debug flags (viper_config.flags). */
-enum { VIPER_FLAG_TIMING = 2 };  /* record CUDA events around the pack / install
+enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install
                                     kernels on their launch streams; the device
                                     times appear in viper_stats (bench.py)       */
+       VIPER_FLAG_NO_FUSE = 4 }; /* producer: never use the fused SYNC kernel
+                                    (pack and install as separate kernels)      */
 
 typedef struct {
     int32_t tier;            /* VIPER_TIER_*                       (default GPU)    */
@@ -204,15 +206,18 @@ typedef struct {
     double writer_wait_us;     /* consumer: time waiting for readers to leave a slot  */
     double t_pack_dev_us;      /* producer, VIPER_FLAG_TIMING: last pack_seal kernel (CUDA events) */
     double t_install_dev_us;   /* consumer, VIPER_FLAG_TIMING: last install_verify kernel          */
+    double t_fused_dev_us;     /* producer, VIPER_FLAG_TIMING: last publish_fused kernel (SYNC,
+                                  in-process: pack + install + verify + swap in one launch)     */
     int32_t last_status;
     int32_t nconsumers;
 } viper_stats;
 viper_status viper_get_stats(viper_model *m, viper_stats *out);
 
 /* Layout queries (for tests / tooling): packed size, per-tensor offsets
- * (offsets may be NULL), and a device pointer to the seal array of the most
- * recent snapshot (producer) or the staged seals (consumer): 2 x uint64
- * {version, cks} per chunk. */
+ * (offsets may be NULL).  viper_debug_buffers: producer -> device pointers of
+ * the most recent snapshot and of its chunk seals (2 x uint64 {version, cks}
+ * per chunk, R16; waits until they are reduced); consumer -> its
+ * DRAM-tier staging buffer (NULL on the GPU tier) and NULL seals. */
 viper_status viper_layout(viper_model *m, uint64_t *s_packed, uint64_t *offsets, int32_t n);
 viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_seals, uint64_t *nchunks);
 

@@ -13,8 +13,12 @@
 //                  atomically" (s4.2 P:1214-1227) -> this is t_c.
 //
 // Both are warp-per-work-item streaming kernels: 128-bit loads/stores, U
-// vectors in flight per lane, one persistent-ish grid sized to the SM count.
-// HBM-bound: algorithmic bytes per launch = 2 * (sum of tensor bytes).
+// vectors in flight per lane, a grid of at most 2 blocks per SM.  HBM-bound:
+// algorithmic bytes per launch = 2 * (sum of tensor bytes).  Checksums are
+// carried per work item (item seal = cks + version * kVerMix) so neither kernel
+// needs a cross-block reduction on its critical path; the chunk seals
+// {version, cks} of DESIGN.md R16 are reduced from them by seal_reduce on a
+// side stream.
 #include "vp_internal.h"
 
 namespace vp {
@@ -33,12 +37,31 @@ __device__ __forceinline__ uint4 ld_stream(const void *p) {
     return r;
 }
 
+__device__ __forceinline__ uint4 ld_cg(const void *p) {  // L2-coherent (data written during this grid)
+    uint4 r;
+    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p));
+    return r;
+}
+
+__device__ __forceinline__ void st_release(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t ld_acquire(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ void st_v4(void *p, const uint4 &v) {
     asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
                  : "memory");
 }
 
-// sum over the 4 words of a 16-B vector whose first word has global index g
+// CKS terms of the 4 words of a 16-B vector whose first word has global index g:
+// sum_k w_k * ((2(g+k)+1) * K) mod 2^32   (R16)
 __device__ __forceinline__ uint64_t cks_vec(const uint4 &v, uint32_t g) {
     const uint32_t m0 = (2u * g + 1u) * kCksK;
     const uint32_t d = 2u * kCksK;
@@ -54,6 +77,7 @@ __device__ __forceinline__ uint64_t warp_sum(uint64_t x) {
 
 // Copy bytes [b0, n) of an item word by word (any alignment); words are
 // little-endian u32 of the packed buffer, zero-extended past n.
+template <bool kCoherent>
 __device__ __forceinline__ uint64_t copy_words_bytewise(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst,
                                                         uint32_t b0, uint32_t n, uint64_t p0, uint32_t lane,
                                                         bool inject_first) {
@@ -62,13 +86,13 @@ __device__ __forceinline__ uint64_t copy_words_bytewise(const uint8_t *__restric
         uint32_t word = 0;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            uint32_t b = w * 4 + k;
-            if (b < n) word |= (uint32_t)src[b] << (8 * k);
+            const uint32_t b = w * 4 + k;
+            if (b < n) word |= (uint32_t)(kCoherent ? __ldcg(src + b) : src[b]) << (8 * k);
         }
         if (inject_first && w * 4 == b0) word ^= 0x10u;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            uint32_t b = w * 4 + k;
+            const uint32_t b = w * 4 + k;
             if (b < n) dst[b] = (uint8_t)(word >> (8 * k));
         }
         const uint32_t g = (uint32_t)((p0 + w * 4) >> 2);
@@ -79,11 +103,12 @@ __device__ __forceinline__ uint64_t copy_words_bytewise(const uint8_t *__restric
 
 // Copy one work item (src -> dst, n bytes, packed offset p0); returns the
 // lane's partial checksum of the packed-space words it moved.
+template <bool kCoherent>
 __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst, uint32_t n,
                                               uint64_t p0, uint32_t lane, bool inject) {
     uint64_t acc = 0;
     const bool aligned = (((uintptr_t)src | (uintptr_t)dst) & 15u) == 0;
-    if (!aligned) return copy_words_bytewise(src, dst, 0, n, p0, lane, inject);
+    if (!aligned) return copy_words_bytewise<kCoherent>(src, dst, 0, n, p0, lane, inject);
     const uint32_t nvec = n >> 4;
     const uint32_t g0 = (uint32_t)(p0 >> 2);
     for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
@@ -91,7 +116,7 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
 #pragma unroll
         for (int u = 0; u < kUnroll; u++) {
             const uint32_t i = base + u * 32 + lane;
-            if (i < nvec) r[u] = ld_stream(src + (size_t)i * 16);
+            if (i < nvec) r[u] = kCoherent ? ld_cg(src + (size_t)i * 16) : ld_stream(src + (size_t)i * 16);
         }
         if (inject && base == 0 && lane == 0) r[0].x ^= 0x10u;
 #pragma unroll
@@ -103,84 +128,216 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
             }
         }
     }
-    if (n & 15u) acc += copy_words_bytewise(src, dst, nvec * 16, n, p0, lane, inject && nvec == 0);
+    if (n & 15u) acc += copy_words_bytewise<kCoherent>(src, dst, nvec * 16, n, p0, lane, inject && nvec == 0);
     return acc;
 }
 
-template <bool kPack>
-__device__ __forceinline__ void finish_item(const Item &it, uint64_t lane_acc, uint32_t lane, const Scratch &s,
-                                            Seal *seals_out, const Seal *seals_in, uint64_t version,
-                                            uint32_t nchunks, bool *last_chunk) {
-    const uint64_t item_cks = warp_sum(lane_acc);
-    *last_chunk = false;
-    if (lane == 0) {
-        const uint32_t c = it.chunk;
-        atomicAdd((unsigned long long *)&s.acc[c], (unsigned long long)item_cks);
-        __threadfence();
-        const uint32_t prev = atomicAdd(&s.cnt[c], 1u);
-        if (prev == it.chunk_items - 1) {
-            __threadfence();
-            const uint64_t total = atomicExch((unsigned long long *)&s.acc[c], 0ull);
-            s.cnt[c] = 0;
-            if (kPack) {
-                volatile Seal *so = seals_out + c;
-                so->cks = total;
-                __threadfence();
-                so->version = version;
-            } else {
-                const volatile Seal *si = seals_in + c;
-                const uint64_t ev = si->version, ec = si->cks;
-                if (ev != version) atomicOr(s.err, kErrVersion);
-                else if (ec != total) atomicOr(s.err, kErrChecksum);
+// Fused copy for the SYNC in-process publish: per U-vector step, stream the
+// tensor piece into the snapshot, immediately read those snapshot bytes back
+// (same lane, same addresses -> ordered; an L2 hit), and store them into each
+// consumer's slot.  Returns the pack checksum; cks_c[k] is the checksum of
+// what consumer k received (the read-back, after any injected fault).
+__device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ src, uint8_t *__restrict__ snap,
+                                                    const uint64_t *dst, uint32_t ncons, uint32_t n, uint64_t p0,
+                                                    uint32_t lane, uint32_t inject_mask, uint64_t *cks_c) {
+    uint64_t acc = 0;
+    bool aligned = (((uintptr_t)src | (uintptr_t)snap) & 15u) == 0;
+#pragma unroll
+    for (int k = 0; k < kMaxFused; k++)
+        if (k < (int)ncons) aligned &= (dst[k] & 15u) == 0;
+    if (!aligned) {  // rare: word path, pack then one read-back per consumer
+        acc = copy_words_bytewise<false>(src, snap, 0, n, p0, lane, false);
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < kMaxFused; k++)
+            if (k < (int)ncons)
+                cks_c[k] += copy_words_bytewise<true>(snap, (uint8_t *)dst[k], 0, n, p0, lane, (inject_mask >> k) & 1u);
+        return acc;
+    }
+    const uint32_t nvec = n >> 4;
+    const uint32_t g0 = (uint32_t)(p0 >> 2);
+    for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
+        uint4 r[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            const uint32_t i = base + u * 32 + lane;
+            if (i < nvec) r[u] = ld_stream(src + (size_t)i * 16);
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            const uint32_t i = base + u * 32 + lane;
+            if (i < nvec) {
+                st_v4(snap + (size_t)i * 16, r[u]);
+                acc += cks_vec(r[u], g0 + 4u * i);
             }
-            __threadfence();
-            const uint32_t d = atomicAdd(s.done, 1u);
-            *last_chunk = (d == nchunks - 1);
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {  // read back what this lane stored
+            const uint32_t i = base + u * 32 + lane;
+            if (i < nvec) r[u] = ld_cg(snap + (size_t)i * 16);
+        }
+#pragma unroll
+        for (int k = 0; k < kMaxFused; k++) {
+            if (k >= (int)ncons) break;
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) {
+                    uint4 x = r[u];
+                    if (u == 0 && base == 0 && lane == 0 && ((inject_mask >> k) & 1u)) x.x ^= 0x10u;
+                    st_v4((uint8_t *)dst[k] + (size_t)i * 16, x);
+                    cks_c[k] += cks_vec(x, g0 + 4u * i);
+                }
+            }
+        }
+    }
+    if (n & 15u) {
+        acc += copy_words_bytewise<false>(src, snap, nvec * 16, n, p0, lane, false);
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < kMaxFused; k++)
+            if (k < (int)ncons)
+                cks_c[k] += copy_words_bytewise<true>(snap, (uint8_t *)dst[k], nvec * 16, n, p0, lane,
+                                                      ((inject_mask >> k) & 1u) && nvec == 0);
+    }
+    return acc;
+}
+
+// pack: stream every item tensor -> packed, write its item seal.  No atomics,
+// no fences: the consumer's kernel is ordered after this one by the stream /
+// event, which makes every store visible.
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_kernel(const PackArgs a) {
+    // let a programmatically-dependent install grid start now: it consumes
+    // items as their ready flags flip (item-granular pack -> install pipeline)
+    asm volatile("griddepcontrol.launch_dependents;");
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        const uint64_t part = warp_sum(copy_item<false>((const uint8_t *)it.ptr, a.packed + it.packed_off,
+                                                        it.nbytes, it.packed_off, lane, false));
+        __syncwarp();  // every lane's stores are ordered before lane 0's release
+        if (lane == 0) {
+            a.iseal[w].mixed = part + a.version * kVerMix;
+            st_release(&a.iseal[w].version, a.version);  // item w ready (pipelined install)
         }
     }
 }
 
-__device__ __forceinline__ void finalize_install(const InstallArgs &a) {
-    __threadfence();
-    const uint32_t e = atomicExch(a.s.err, 0u);
-    *a.s.done = 0;
-    const int32_t st = (e & kErrVersion) ? -4 : ((e & kErrChecksum) ? -5 : 0);
-    if (a.status_h) *a.status_h = st;
-    __threadfence_system();
-    if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
-    if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
-    __threadfence_system();
-}
-
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_kernel(const PackArgs a) {
+// chunk seals {version, sum of item checksums} -- one warp per chunk, off the
+// critical path (side stream); they are what DESIGN.md R16 / the oracle define.
+__global__ void seal_reduce_kernel(const SealReduceArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t warps = gridDim.x * (blockDim.x >> 5);
-    for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < a.nitems; w += warps) {
-        const Item it = a.items[w];
-        const uint8_t *src = a.src[it.tensor] + it.tensor_off;
-        uint8_t *dst = a.packed + it.packed_off;
-        const uint64_t acc = copy_item(src, dst, it.nbytes, it.packed_off, lane, false);
-        bool last;
-        finish_item<true>(it, acc, lane, a.s, a.seals, nullptr, a.version, a.nchunks, &last);
-        if (lane == 0 && last) *a.s.done = 0;  // every chunk sealed: reset for the next launch
+    const uint32_t c = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    if (c >= a.nchunks) return;
+    const uint32_t lo = a.chunk_first[c], hi = a.chunk_first[c + 1];
+    uint64_t s = 0;
+    for (uint32_t i = lo + lane; i < hi; i += 32) s += a.iseal[i].mixed - a.version * kVerMix;
+    s = warp_sum(s);
+    if (lane == 0) {
+        a.seals[c].cks = s;
+        a.seals[c].version = a.version;
     }
 }
 
+// install: stream every item packed -> slot tensor, recompute its seal and
+// compare with the producer's; the last block to finish publishes the result
+// and, if every item matched, swaps the version word from the device.
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_verify_kernel(const InstallArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
-    if (a.nitems == 0) {  // empty model: nothing to copy, still swap
-        if (blockIdx.x == 0 && threadIdx.x == 0) finalize_install(a);
-        return;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    bool bad = false;
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    Item it{};
+    if (w < a.nitems) it = a.items[w];
+    for (; w < a.nitems; w += nwarps) {
+        if (w >= blockIdx.x * kWarpsPerBlock + nwarps) it = a.items[w];
+        // Item-granular pipeline: with PDL the install grid runs concurrently
+        // with the pack grid (all of whose blocks are resident by then, so
+        // this cannot deadlock); wait for item w's ready flag, then stream it
+        // with L2-coherent loads.  Without PDL the flag is already set.
+        uint64_t expect = 0;
+        if (lane == 0) {
+            const ISeal *is = a.iseal + w;
+            uint32_t backoff = 32;
+            while (ld_acquire(&is->version) != a.version) {
+                __nanosleep(backoff);
+                if (backoff < 1024) backoff <<= 1;
+            }
+            expect = is->mixed;
+        }
+        __syncwarp();
+        const uint64_t part = warp_sum(copy_item<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes,
+                                                       it.packed_off, lane, w == a.fault_item));
+        if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
     }
-    const uint32_t warps = gridDim.x * (blockDim.x >> 5);
-    for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < a.nitems; w += warps) {
+    if (bad) atomicOr(a.err, kErrChecksum);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();  // cumulative over the block's stores (ordered by the barrier)
+        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
+            __threadfence();
+            const uint32_t e = atomicExch(a.err, 0u);
+            *a.done = 0;
+            const int32_t st = (e & kErrChecksum) ? -5 : 0;
+            // Every block's slot stores are GPU-visible (cumulative fences
+            // above); later readers are kernels launched after the host saw
+            // the flip, so plain system-visible stores suffice here.
+            if (a.status_h) *a.status_h = st;
+            if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
+            if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
+        }
+    }
+}
+
+// SYNC in-process publish, pack + install fused per warp.  Lane l re-reads
+// exactly the snapshot bytes it stored (same thread, so ordered) with L2
+// loads, installs them and recomputes the item checksum; the seal check is
+// against the value just sealed.  No cross-warp dependency inside the grid.
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fused_kernel(const FusedArgs a) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    uint32_t bad = 0;
+    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
         const Item it = a.items[w];
-        const uint8_t *src = a.packed + it.packed_off;
-        uint8_t *dst = a.dst[it.tensor] + it.tensor_off;
-        const uint64_t acc = copy_item(src, dst, it.nbytes, it.packed_off, lane, w == a.fault_item);
-        bool last;
-        finish_item<false>(it, acc, lane, a.s, nullptr, a.seals, a.version, a.nchunks, &last);
-        if (lane == 0 && last) finalize_install(a);
+        uint64_t cptr[kMaxFused];  // only the slot address differs between the lists
+        uint32_t inject = 0;
+#pragma unroll
+        for (int k = 0; k < kMaxFused; k++) {
+            cptr[k] = k < (int)a.ncons ? a.cons[k].items[w].ptr : 0;
+            if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
+        }
+        uint64_t got[kMaxFused] = {0, 0, 0, 0};
+        const uint64_t part = warp_sum(copy_item_fused((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
+                                                       a.ncons, it.nbytes, it.packed_off, lane, inject, got));
+        const uint64_t sealed = part + a.version * kVerMix;
+        __syncwarp();
+        if (lane == 0) {
+            a.iseal[w].mixed = sealed;
+            st_release(&a.iseal[w].version, a.version);
+        }
+#pragma unroll
+        for (int k = 0; k < kMaxFused; k++) {
+            if (k >= (int)a.ncons) break;
+            if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
+        }
+    }
+    if (lane == 0 && bad) atomicOr(a.err, bad);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
+            __threadfence();
+            const uint32_t e = atomicExch(a.err, 0u);
+            *a.done = 0;
+            for (uint32_t k = 0; k < a.ncons; k++) {
+                const FusedCons &c = a.cons[k];
+                const int32_t st = (e >> k) & 1u ? -5 : 0;
+                if (c.status_h) *c.status_h = st;
+                if (st == 0 && c.state_h) *c.state_h = (a.version << 1) | (uint64_t)c.target;  // the swap
+                if (c.pin_h) *c.pin_h = 0;
+            }
+        }
     }
 }
 
@@ -205,9 +362,28 @@ cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st) {
-    install_verify_kernel<<<g.grid, g.block, 0, st>>>(a);
+cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
+    publish_fused_kernel<<<g.grid, g.block, 0, st>>>(a);
     return cudaGetLastError();
+}
+
+cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st) {
+    if (a.nchunks == 0) return cudaSuccess;
+    seal_reduce_kernel<<<(a.nchunks + 7) / 8, 256, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl) {
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(g.grid);
+    cfg.blockDim = dim3(g.block);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, install_verify_kernel, a);
 }
 
 }  // namespace vp

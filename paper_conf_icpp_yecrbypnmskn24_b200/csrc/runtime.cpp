@@ -23,6 +23,7 @@
 
 namespace vp {
 
+extern int64_t g_trace[16];
 static thread_local std::string t_err;
 
 viper_status set_error(viper_status st, const char *fmt, ...) {
@@ -86,51 +87,50 @@ static viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n
     m.nchunks = (uint32_t)((m.s_packed + chunk_bytes - 1) / chunk_bytes);
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    // item size: enough items for ~4 per resident warp, 2 KiB .. 64 KiB, 512-B multiple
+    // item size: enough items for ~4 per resident warp, 2 KiB .. 16 KiB, 512-B
+    // multiple.  The 16 KiB cap keeps the fused kernel's read-back window
+    // (resident warps x item) at ~77 MB, inside the 126 MB L2.
     uint64_t target = m.s_packed / ((uint64_t)sms * 32 * 4) + 1;
-    uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), 65536);
+    uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), 16384);
     if (item_max > chunk_bytes) item_max = chunk_bytes;
     m.items.clear();
     std::vector<uint32_t> per_chunk(m.nchunks, 0);
     for (int32_t i = 0; i < n; i++) {
         uint64_t done = 0;
         while (done < m.nbytes[i]) {
-            uint64_t p = m.offsets[i] + done;
-            uint64_t chunk = p / chunk_bytes;
-            uint64_t chunk_end = (chunk + 1) * chunk_bytes;
-            uint64_t len = std::min<uint64_t>({item_max, m.nbytes[i] - done, chunk_end - p});
-            Item it{};
-            it.packed_off = p;
-            it.tensor_off = done;
-            it.nbytes = (uint32_t)len;
-            it.tensor = (uint32_t)i;
-            it.chunk = (uint32_t)chunk;
-            m.items.push_back(it);
+            const uint64_t p = m.offsets[i] + done;
+            const uint64_t chunk = p / chunk_bytes;
+            const uint64_t chunk_end = (chunk + 1) * chunk_bytes;
+            const uint64_t len = std::min<uint64_t>({item_max, m.nbytes[i] - done, chunk_end - p});
+            m.items.push_back(BaseItem{done, p, (uint32_t)len, (uint32_t)chunk, (uint32_t)i});
             per_chunk[chunk]++;
             done += len;
         }
     }
-    for (uint32_t c = 0; c < m.nchunks; c++)
+    m.chunk_first.assign(m.nchunks + 1, 0);
+    for (uint32_t c = 0; c < m.nchunks; c++) {
         if (per_chunk[c] == 0) return set_error(VIPER_E_INVAL, "chunk %u has no data (align > chunk?)", c);
-    for (auto &it : m.items) it.chunk_items = per_chunk[it.chunk];
-    if (m.items.size() >= (size_t)UINT32_MAX) return set_error(VIPER_E_INVAL, "too many work items");
-    if (!m.items.empty()) {
-        CUDA_TRY(cudaMalloc(&m.d_items, m.items.size() * sizeof(Item)));
-        CUDA_TRY(cudaMemcpy(m.d_items, m.items.data(), m.items.size() * sizeof(Item), cudaMemcpyHostToDevice));
+        m.chunk_first[c + 1] = m.chunk_first[c] + per_chunk[c];
     }
+    if (m.items.size() >= (size_t)UINT32_MAX) return set_error(VIPER_E_INVAL, "too many work items");
+    CUDA_TRY(cudaMalloc(&m.d_chunk_first, m.chunk_first.size() * sizeof(uint32_t)));
+    CUDA_TRY(cudaMemcpy(m.d_chunk_first, m.chunk_first.data(), m.chunk_first.size() * sizeof(uint32_t),
+                        cudaMemcpyHostToDevice));
     return VIPER_OK;
 }
 
-static viper_status alloc_scratch(viper_model *m) {
-    const size_t nch = m->man.nchunks ? m->man.nchunks : 1;
-    const size_t bytes = nch * sizeof(uint64_t) + nch * sizeof(uint32_t) + 64;
-    CUDA_TRY(cudaMalloc(&m->scratch_alloc, bytes));
-    CUDA_TRY(cudaMemset(m->scratch_alloc, 0, bytes));
-    uint8_t *p = (uint8_t *)m->scratch_alloc;
-    m->scratch.acc = (uint64_t *)p;
-    m->scratch.cnt = (uint32_t *)(p + nch * sizeof(uint64_t));
-    m->scratch.done = (uint32_t *)(p + nch * sizeof(uint64_t) + nch * sizeof(uint32_t));
-    m->scratch.err = m->scratch.done + 4;
+// Device work list of one endpoint: the base items with that endpoint's tensor
+// addresses folded in.
+static viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out) {
+    *d_out = nullptr;
+    if (m.items.empty()) return VIPER_OK;
+    std::vector<Item> v(m.items.size());
+    for (size_t k = 0; k < v.size(); k++) {
+        const BaseItem &b = m.items[k];
+        v[k] = Item{(uint64_t)(uintptr_t)ptrs[b.tensor] + b.tensor_off, b.packed_off, b.nbytes, b.chunk, b.tensor, 0};
+    }
+    CUDA_TRY(cudaMalloc((void **)d_out, v.size() * sizeof(Item)));
+    CUDA_TRY(cudaMemcpy(*d_out, v.data(), v.size() * sizeof(Item), cudaMemcpyHostToDevice));
     return VIPER_OK;
 }
 
@@ -202,64 +202,79 @@ static bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
     }
 }
 
-// Enqueue the install of snapshot slot b (version v) of producer p into the
-// inactive slot of consumer c on stream st.  Caller holds c->install_mu and
-// has pinned v.  wait_ready: make st wait for the producer's snapshot event.
-static viper_status enqueue_install(viper_model *c, viper_model *p, uint64_t v, int b, cudaStream_t st,
-                                    bool wait_ready) {
+struct PreparedInstall {
+    viper_model *c = nullptr;
+    InstallArgs a{};
+    double waited_us = 0;
+};
+
+// Host half of an install of snapshot slot b (version v) of producer p into
+// the inactive slot of consumer c: wait until no reader pins the target (a7)
+// and build the kernel arguments.  Caller holds c->install_mu.
+static viper_status prepare_install(viper_model *c, viper_model *p, uint64_t v, int b, PreparedInstall *pi) {
     ConsRec *r = c->rec;
     const uint64_t cur = r->state.load();
     const int target = cur == 0 ? 0 : (int)(1 - (cur & 1));
-    // The alternative copy is written only when no reader pins it (a7).
     const int64_t t0 = now_ns();
     while (r->ref[target].load() != 0) {
         if (now_ns() - t0 > 10ll * 1000000000ll)
             return set_error(VIPER_E_TIMEOUT, "readers kept slot %d pinned for 10 s", target);
         sched_yield();
     }
-    const double waited = (now_ns() - t0) / 1e3;
-    const uint8_t *src;
-    const Seal *seals;
-    if (wait_ready) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
-    if (c->cfg.tier == VIPER_TIER_DRAM) {
-        // Host-to-Host channel (P:1697-1720): host staging -> this GPU's staging
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage, p->h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage_seals, p->h_seal[b], sizeof(Seal) * c->man.nchunks,
-                                 cudaMemcpyHostToDevice, st));
-        src = c->d_stage;
-        seals = c->d_stage_seals;
-    } else {
-        src = p->d_snap[b];
-        seals = p->d_seal[b];
-    }
-    InstallArgs a{};
-    a.items = c->man.d_items;
+    pi->c = c;
+    pi->waited_us = (now_ns() - t0) / 1e3;
+    InstallArgs &a = pi->a;
+    a = InstallArgs{};
+    const bool dram = c->cfg.tier == VIPER_TIER_DRAM;
+    a.items = c->d_slot_items[target];
     a.nitems = (uint32_t)c->man.items.size();
-    a.nchunks = c->man.nchunks;
-    a.dst = c->d_slot[target];
-    a.packed = src;
-    a.seals = seals;
-    a.s = c->scratch;
+    a.packed = dram ? c->d_stage : p->d_snap[b];
+    a.iseal = dram ? c->d_stage_iseal : p->d_iseal[b];
     a.version = v;
     a.target = (uint32_t)target;
     a.fault_item = ~0u;
     if (c->fault_next.exchange(false) && a.nitems) a.fault_item = a.nitems / 2;
+    a.done = c->d_flags;
+    a.err = c->d_flags + 1;
     a.status_h = (volatile int32_t *)&c->rec_dev->status;
     a.pin_h = (volatile uint64_t *)&c->rec_dev->pin;
     a.state_h = (volatile uint64_t *)&c->rec_dev->state;
-    r->status.store(1);  // "in flight"
+    return VIPER_OK;
+}
+
+// Stream half: [wait for the snapshot] [DRAM tier: H2D staging] install kernel.
+// pdl: the kernel directly follows the pack on st and consumes its items as
+// they are sealed (kernels.cu, item-granular pipeline).
+static viper_status launch_prepared(PreparedInstall &pi, viper_model *p, int b, cudaStream_t st, bool wait_ready,
+                                    bool pdl) {
+    viper_model *c = pi.c;
+    if (wait_ready) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
+    if (c->cfg.tier == VIPER_TIER_DRAM) {
+        // Host-to-Host channel (P:1697-1720): host staging -> this GPU's staging
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, p->h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, p->h_iseal[b], sizeof(ISeal) * c->man.items.size(),
+                                 cudaMemcpyHostToDevice, st));
+        pdl = false;
+    }
+    c->rec->status.store(1);  // "in flight"
     const bool timing = c->cfg.flags & VIPER_FLAG_TIMING;
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
-    CUDA_TRY(launch_install(a, c->geo, st));
+    CUDA_TRY(launch_install(pi.a, c->geo, st, pdl && !timing));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
         c->timing_pending = true;
     }
-    {
-        std::lock_guard<std::mutex> lk(c->stats_mu);
-        c->stats.writer_wait_us = waited;
-    }
+    std::lock_guard<std::mutex> lk(c->stats_mu);
+    c->stats.writer_wait_us = pi.waited_us;
     return VIPER_OK;
+}
+
+static viper_status enqueue_install(viper_model *c, viper_model *p, uint64_t v, int b, cudaStream_t st,
+                                    bool wait_ready) {
+    PreparedInstall pi;
+    viper_status s = prepare_install(c, p, v, b, &pi);
+    if (s) return s;
+    return launch_prepared(pi, p, b, st, wait_ready, false);
 }
 
 // After the install kernel of v completed on the host's view of the stream.
@@ -268,7 +283,8 @@ static viper_status finish_install(viper_model *c, uint64_t v, double t_install_
     viper_status st = r->status.load();
     if (st == 1) st = set_error(VIPER_E_CUDA, "install kernel did not report");
     float dev_ms = -1.f;
-    if (c->timing_pending && cudaEventElapsedTime(&dev_ms, c->ev_t[0], c->ev_t[1]) == cudaSuccess)
+    if (c->timing_pending && cudaEventSynchronize(c->ev_t[1]) == cudaSuccess &&
+        cudaEventElapsedTime(&dev_ms, c->ev_t[0], c->ev_t[1]) == cudaSuccess)
         c->timing_pending = false;
     {
         std::lock_guard<std::mutex> lk(c->stats_mu);
@@ -286,7 +302,7 @@ static viper_status finish_install(viper_model *c, uint64_t v, double t_install_
     r->last_status.store(st);
     r->done_version.store(v);
     r->done_seq.fetch_add(1);
-    futex_wake_all(&r->done_seq);
+    if (r->waiters.load() > 0) futex_wake_all(&r->done_seq);
     return st;
 }
 
@@ -357,8 +373,36 @@ static void update_loop(viper_model *c) {
 }
 
 // ------------------------------------------------------------------ producer
+// Wait until consumer c's install of v reported (mapped status word), without
+// a stream synchronisation: the install kernel's last block writes status and
+// then the version word.
+static viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
+    ConsRec *r = c->rec;
+    const int64_t t0 = now_ns();
+    for (uint32_t spins = 0;; spins++) {
+        const int32_t s = r->status.load();
+        if (s != 1) {
+            if (s == VIPER_OK)
+                while ((r->state.load() >> 1) != v) cpu_relax();
+            return VIPER_OK;
+        }
+        if ((spins & 1023) == 1023) {
+            const cudaError_t q = cudaStreamQuery(st);  // surfaces launch / device errors
+            if (q != cudaSuccess && q != cudaErrorNotReady)
+                return set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(q));
+            if (q == cudaSuccess && r->status.load() == 1) return set_error(VIPER_E_CUDA, "install kernel did not report");
+            if (now_ns() - t0 > 60ll * 1000000000ll) return set_error(VIPER_E_TIMEOUT, "install did not finish");
+        }
+        cpu_relax();
+    }
+}
+
+int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug_trace)
+#define TRACE(i) (g_trace[i] = now_ns())
+
 static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st) {
     const int64_t t0 = now_ns();
+    g_trace[0] = t0;
     if (v == 0 || v <= p->last_version)
         return set_error(VIPER_E_VERSION, "publish(%llu) after %llu: versions strictly increase from 1",
                          (unsigned long long)v, (unsigned long long)p->last_version);
@@ -381,74 +425,139 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         }
         // the DRAM-tier D2H of old_v must be finished before overwriting
         if (p->cfg.tier == VIPER_TIER_DRAM) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
+        // ... and so must the side-stream seal reduction reading its item seals
+        CUDA_TRY(cudaStreamWaitEvent(st, p->ev_sealed[b], 0));
     }
-    PackArgs a{};
-    a.items = p->man.d_items;
-    a.nitems = (uint32_t)p->man.items.size();
-    a.nchunks = p->man.nchunks;
-    a.src = p->d_src;
-    a.packed = p->d_snap[b];
-    a.seals = p->d_seal[b];
-    a.s = p->scratch;
-    a.version = v;
-    const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
-    if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
-    CUDA_TRY(launch_pack(a, p->geo, st));
-    if (timing) {
-        CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
-        p->timing_pending = true;
-    }
-    if (p->cfg.tier == VIPER_TIER_DRAM) {
-        // snapshot -> pinned host, on a side stream so the
-        // caller's stream is blocked only by the pack
-        CUDA_TRY(cudaEventRecord(p->ev_packed, st));
-        CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
-        CUDA_TRY(cudaMemcpyAsync(p->h_stage[b], p->d_snap[b], p->man.s_packed, cudaMemcpyDeviceToHost, p->side));
-        CUDA_TRY(cudaMemcpyAsync(p->h_seal[b], p->d_seal[b], sizeof(Seal) * p->man.nchunks,
-                                 cudaMemcpyDeviceToHost, p->side));
-        CUDA_TRY(cudaEventRecord(p->ev_ready[b], p->side));
-    } else {
-        CUDA_TRY(cudaEventRecord(p->ev_ready[b], st));
-    }
-    p->snap_version[b] = v;
-    p->cur_snap = b;
-    p->last_version = v;
-    ctrl->pub_state.store((v << 1) | (uint64_t)b);
-    ctrl->pub_time_ns.store(now_ns());
-
+    TRACE(1);
+    const bool dram = p->cfg.tier == VIPER_TIER_DRAM;
+    const bool sync = p->cfg.mode == VIPER_SYNC;
     viper_status result = VIPER_OK;
-    if (p->cfg.mode == VIPER_SYNC) {
-        // SYNC: deliver + install inline, stream-ordered after the
-        // pack; return once every consumer swapped (or failed).
+    // SYNC: this thread delivers + installs for every local
+    // consumer, then returns once each swapped (or failed).  The host half of
+    // each install (reader wait, arguments) is done BEFORE the pack launch so
+    // that the first install lands right behind it on the stream (PDL).  The
+    // producer waits for these installs itself, so no snapshot pin is needed.
+    std::vector<std::unique_lock<std::mutex>> locks;
+    std::vector<PreparedInstall> prepared;
+    if (sync) {
         std::vector<viper_model *> cons;
         {
             std::lock_guard<std::mutex> lk(g_reg_mu);
             cons = p->chan->consumers;
         }
-        std::vector<std::unique_lock<std::mutex>> locks;
-        std::vector<viper_model *> launched;
         for (viper_model *c : cons) {
             std::unique_lock<std::mutex> lk(c->install_mu);
-            if (c->attempted >= v) continue;  // its update thread already did v
-            uint64_t pv;
-            int pb;
-            if (!pin_latest(ctrl, c->rec, &pv, &pb) || pv != v) continue;
-            c->attempted = v;
-            viper_status s = enqueue_install(c, p, v, b, st, p->cfg.tier == VIPER_TIER_DRAM);
+            if (c->attempted >= v) continue;
+            PreparedInstall pi;
+            viper_status s = prepare_install(c, p, v, b, &pi);
             if (s != VIPER_OK) {
-                c->rec->pin.store(0);
                 result = s;
                 continue;
             }
-            launched.push_back(c);
+            c->attempted = v;
+            prepared.push_back(pi);
             locks.push_back(std::move(lk));
         }
+    }
+    TRACE(2);
+    const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
+    std::vector<viper_model *> launched;
+    const bool fuse = sync && !dram && !prepared.empty() && prepared.size() <= (size_t)kMaxFused &&
+                      !(p->cfg.flags & VIPER_FLAG_NO_FUSE);
+    if (fuse) {
+        // one kernel: pack + seal + install + verify + swap for every local consumer
+        FusedArgs f{};
+        f.items = p->d_items;
+        f.nitems = (uint32_t)p->man.items.size();
+        f.ncons = (uint32_t)prepared.size();
+        f.packed = p->d_snap[b];
+        f.iseal = p->d_iseal[b];
+        f.version = v;
+        f.done = p->d_flags;
+        f.err = p->d_flags + 1;
+        for (size_t k = 0; k < prepared.size(); k++) {
+            const InstallArgs &ia = prepared[k].a;
+            f.cons[k] = FusedCons{ia.items, ia.target, ia.fault_item, ia.status_h, ia.pin_h, ia.state_h};
+            prepared[k].c->rec->status.store(1);
+            std::lock_guard<std::mutex> lk(prepared[k].c->stats_mu);
+            prepared[k].c->stats.writer_wait_us = prepared[k].waited_us;
+        }
+        if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
+        CUDA_TRY(launch_fused(f, p->geo, st));
+        if (timing) {
+            CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
+            p->timing_pending = true;
+        }
+        for (PreparedInstall &pi : prepared) launched.push_back(pi.c);
+        prepared.clear();
+    } else {
+        PackArgs a{};
+        a.items = p->d_items;
+        a.nitems = (uint32_t)p->man.items.size();
+        a.packed = p->d_snap[b];
+        a.iseal = p->d_iseal[b];
+        a.version = v;
+        if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
+        CUDA_TRY(launch_pack(a, p->geo, st));
+        if (timing) {
+            CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
+            p->timing_pending = true;
+        }
+    }
+    p->last_fused = fuse;
+    auto launch_all = [&]() {
+        for (PreparedInstall &pi : prepared) {
+            viper_status s = launch_prepared(pi, p, b, st, dram, !dram && launched.empty());
+            if (s != VIPER_OK) {
+                result = s;
+                continue;
+            }
+            launched.push_back(pi.c);
+        }
+    };
+    if (sync && !dram) launch_all();
+    TRACE(3);
+    if (!dram) CUDA_TRY(cudaEventRecord(p->ev_ready[b], st));
+    p->snap_version[b] = v;
+    p->cur_snap = b;
+    p->last_version = v;
+    ctrl->pub_state.store((v << 1) | (uint64_t)b);
+    ctrl->pub_time_ns.store(now_ns());
+    // chunk seals (R16) from the item seals, on the side stream
+    CUDA_TRY(cudaEventRecord(p->ev_packed, st));
+    CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
+    SealReduceArgs ra{};
+    ra.chunk_first = p->man.d_chunk_first;
+    ra.nchunks = p->man.nchunks;
+    ra.iseal = p->d_iseal[b];
+    ra.seals = p->d_seal[b];
+    ra.version = v;
+    CUDA_TRY(launch_seal_reduce(ra, p->side));
+    if (dram) {
+        // snapshot -> pinned host on the side stream, so the
+        // caller's stream is blocked only by the pack
+        CUDA_TRY(cudaMemcpyAsync(p->h_stage[b], p->d_snap[b], p->man.s_packed, cudaMemcpyDeviceToHost, p->side));
+        CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b], p->d_iseal[b], sizeof(ISeal) * p->man.items.size(),
+                                 cudaMemcpyDeviceToHost, p->side));
+        CUDA_TRY(cudaEventRecord(p->ev_ready[b], p->side));
+    }
+    CUDA_TRY(cudaEventRecord(p->ev_sealed[b], p->side));
+    TRACE(4);
+    if (sync && dram) launch_all();
+
+    if (sync) {
         const int64_t ti = now_ns();
-        CUDA_TRY(cudaStreamSynchronize(st));
         for (viper_model *c : launched) {
-            viper_status s = finish_install(c, v, (now_ns() - ti) / 1e3);
+            viper_status s = wait_install_done(c, v, st);
+            TRACE(5);
+            if (s != VIPER_OK) {
+                c->rec->status.store(s);
+                if (result == VIPER_OK) result = s;
+            }
+            s = finish_install(c, v, (now_ns() - ti) / 1e3);
             if (s != VIPER_OK && result == VIPER_OK) result = s;
         }
+        TRACE(6);
         locks.clear();
         for (viper_model *c : launched) fire_callback(c, v, c->rec->last_status.load());
     } else {
@@ -461,6 +570,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         p->stats.t_publish_us = (now_ns() - t0) / 1e3;
         p->stats.last_status = result;
     }
+    TRACE(7);
     return result;
 }
 
@@ -472,13 +582,6 @@ static viper_status check_tensors(const viper_tensor *t, int32_t n) {
         if (t[i].dtype < VIPER_F32 || t[i].dtype > VIPER_BYTES) return set_error(VIPER_E_INVAL, "tensor %d: dtype", i);
         if (t[i].nbytes > 0xFFFFFFFFull * 64) return set_error(VIPER_E_INVAL, "tensor %d too large", i);
     }
-    return VIPER_OK;
-}
-
-static viper_status upload_ptrs(const std::vector<void *> &ptrs, void ***d_out) {
-    const size_t bytes = std::max<size_t>(ptrs.size(), 1) * sizeof(void *);
-    CUDA_TRY(cudaMalloc((void **)d_out, bytes));
-    if (!ptrs.empty()) CUDA_TRY(cudaMemcpy(*d_out, ptrs.data(), ptrs.size() * sizeof(void *), cudaMemcpyHostToDevice));
     return VIPER_OK;
 }
 
@@ -504,74 +607,67 @@ static void free_model(viper_model *m) {
         }
         channel_close(m->chan);
     }
-    cudaFree(m->man.d_items);
-    cudaFree(m->scratch_alloc);
-    cudaFree((void *)m->d_src);
+    cudaFree(m->man.d_chunk_first);
+    cudaFree(m->d_items);
+    cudaFree(m->d_slot_items[0]);
+    cudaFree(m->d_slot_items[1]);
+    cudaFree(m->d_flags);
     cudaFree(m->snap_alloc);
-    cudaFree(m->d_slot[0]);
-    cudaFree(m->d_slot[1]);
     cudaFree(m->slot1_alloc);
     cudaFree(m->stage_alloc);
     if (m->h_stage_alloc) cudaFreeHost(m->h_stage_alloc);
-    for (auto &e : m->ev_ready)
-        if (e) cudaEventDestroy(e);
-    for (auto &e : m->ev_t)
-        if (e) cudaEventDestroy(e);
+    for (auto *evs : {m->ev_ready, m->ev_sealed, m->ev_t})
+        for (int k = 0; k < 2; k++)
+            if (evs[k]) cudaEventDestroy(evs[k]);
     if (m->ev_packed) cudaEventDestroy(m->ev_packed);
     if (m->side) cudaStreamDestroy(m->side);
     if (m->ustream) cudaStreamDestroy(m->ustream);
     delete m;
 }
 
-static viper_status register_local(viper_model *m, const viper_tensor *tensors) {
-    viper_status st = channel_open(m->name, m->man, &m->chan);
+static uint64_t al256(uint64_t x) { return (x + 255) / 256 * 256; }
+
+// Producer-side buffers: two snapshot slots (the latest + the one being
+// filled), their item seals and chunk seals, the events and side stream.
+static viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) {
+    const uint64_t S = al256(m->man.s_packed);
+    const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
+    const uint64_t CS = al256(sizeof(Seal) * std::max<uint32_t>(m->man.nchunks, 1));
+    for (int32_t i = 0; i < m->man.n; i++) m->src_ptrs.push_back(tensors[i].dev_ptr);
+    viper_status st = upload_items(m->man, m->src_ptrs, &m->d_items);
     if (st) return st;
-    m->ctrl = m->chan->ctrl;
-    m->ctrl_dev = m->chan->ctrl_dev;
+    const size_t bytes = 2 * (S + IS + CS);
+    CUDA_TRY(cudaMalloc(&m->snap_alloc, bytes));
+    CUDA_TRY(cudaMemset(m->snap_alloc, 0, bytes));  // padding bytes stay 0 forever
+    uint8_t *p = (uint8_t *)m->snap_alloc;
+    for (int b = 0; b < 2; b++) {
+        m->d_snap[b] = p + b * S;
+        m->d_iseal[b] = (ISeal *)(p + 2 * S + b * IS);
+        m->d_seal[b] = (Seal *)(p + 2 * S + 2 * IS + b * CS);
+    }
+    for (auto &e : m->ev_ready) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto &e : m->ev_sealed) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
+    CUDA_TRY(cudaEventCreateWithFlags(&m->ev_packed, cudaEventDisableTiming));
+    CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
+    CUDA_TRY(cudaMalloc(&m->d_flags, 64));
+    CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
+    if (m->cfg.tier == VIPER_TIER_DRAM) {
+        CUDA_TRY(cudaHostAlloc(&m->h_stage_alloc, 2 * (S + IS), cudaHostAllocPortable));
+        uint8_t *h = (uint8_t *)m->h_stage_alloc;
+        for (int b = 0; b < 2; b++) {
+            m->h_stage[b] = h + b * S;
+            m->h_iseal[b] = (ISeal *)(h + 2 * S + b * IS);
+        }
+    }
+    return VIPER_OK;
+}
+
+// Consumer-side buffers: slot 1 (unless supplied), per-slot work lists,
+// completion flags, DRAM-tier staging, the update stream.
+static viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
+    viper_status st;
     const uint64_t S = m->man.s_packed;
-    const size_t seal_bytes = sizeof(Seal) * std::max<uint32_t>(m->man.nchunks, 1);
-    if (m->role == VIPER_PRODUCER) {
-        {
-            std::lock_guard<std::mutex> lk(g_reg_mu);
-            if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
-            m->chan->producer = m;
-        }
-        for (int32_t i = 0; i < m->man.n; i++) m->src_ptrs.push_back(tensors[i].dev_ptr);
-        if ((st = upload_ptrs(m->src_ptrs, (void ***)&m->d_src))) return st;
-        // two snapshot slots (latest + one being filled) + their seals
-        const uint64_t S_al = (S + 255) / 256 * 256;
-        const size_t bytes = 2 * S_al + 2 * seal_bytes;
-        CUDA_TRY(cudaMalloc(&m->snap_alloc, bytes));
-        CUDA_TRY(cudaMemset(m->snap_alloc, 0, bytes));  // padding bytes stay 0 forever
-        m->d_snap[0] = (uint8_t *)m->snap_alloc;
-        m->d_snap[1] = m->d_snap[0] + S_al;
-        m->d_seal[0] = (Seal *)(m->d_snap[1] + S_al);
-        m->d_seal[1] = (Seal *)((uint8_t *)m->d_seal[0] + seal_bytes);
-        for (auto &e : m->ev_ready) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-        for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
-        CUDA_TRY(cudaEventCreateWithFlags(&m->ev_packed, cudaEventDisableTiming));
-        if (m->cfg.tier == VIPER_TIER_DRAM) {
-            CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
-            CUDA_TRY(cudaHostAlloc(&m->h_stage_alloc, 2 * S_al + 2 * seal_bytes, cudaHostAllocPortable));
-            m->h_stage[0] = (uint8_t *)m->h_stage_alloc;
-            m->h_stage[1] = m->h_stage[0] + S_al;
-            m->h_seal[0] = (Seal *)(m->h_stage[1] + S_al);
-            m->h_seal[1] = (Seal *)((uint8_t *)m->h_seal[0] + seal_bytes);
-        }
-        return VIPER_OK;
-    }
-    // consumer
-    {
-        std::lock_guard<std::mutex> lk(g_reg_mu);
-        const int idx = m->ctrl->ncons.load();
-        if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
-        m->cidx = idx;
-        m->rec = &m->ctrl->cons[idx];
-        m->rec_dev = &m->ctrl_dev->cons[idx];
-        m->rec->active.store(1);
-        m->ctrl->ncons.store(idx + 1);
-        m->chan->consumers.push_back(m);
-    }
     for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[0].push_back(tensors[i].dev_ptr);
     if (m->cfg.slot1) {
         for (int32_t i = 0; i < m->man.n; i++) {
@@ -584,14 +680,45 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
         for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[1].push_back((uint8_t *)m->slot1_alloc + m->man.offsets[i]);
     }
     for (int s = 0; s < 2; s++)
-        if ((st = upload_ptrs(m->slot_ptrs[s], (void ***)&m->d_slot[s]))) return st;
+        if ((st = upload_items(m->man, m->slot_ptrs[s], &m->d_slot_items[s]))) return st;
+    CUDA_TRY(cudaMalloc(&m->d_flags, 64));
+    CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
     if (m->cfg.tier == VIPER_TIER_DRAM) {
-        CUDA_TRY(cudaMalloc(&m->stage_alloc, (S + 255) / 256 * 256 + seal_bytes));
+        const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
+        CUDA_TRY(cudaMalloc(&m->stage_alloc, al256(S) + IS));
         m->d_stage = (uint8_t *)m->stage_alloc;
-        m->d_stage_seals = (Seal *)(m->d_stage + (S + 255) / 256 * 256);
+        m->d_stage_iseal = (ISeal *)(m->d_stage + al256(S));
     }
     CUDA_TRY(cudaStreamCreateWithFlags(&m->ustream, cudaStreamNonBlocking));
     for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
+    return VIPER_OK;
+}
+
+static viper_status register_local(viper_model *m, const viper_tensor *tensors) {
+    viper_status st = channel_open(m->name, m->man, &m->chan);
+    if (st) return st;
+    m->ctrl = m->chan->ctrl;
+    m->ctrl_dev = m->chan->ctrl_dev;
+    if (m->role == VIPER_PRODUCER) {
+        {
+            std::lock_guard<std::mutex> lk(g_reg_mu);
+            if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
+            m->chan->producer = m;
+        }
+        return alloc_producer(m, tensors);
+    }
+    if ((st = alloc_consumer(m, tensors))) return st;
+    {
+        std::lock_guard<std::mutex> lk(g_reg_mu);
+        const int idx = m->ctrl->ncons.load();
+        if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+        m->cidx = idx;
+        m->rec = &m->ctrl->cons[idx];
+        m->rec_dev = &m->ctrl_dev->cons[idx];
+        m->rec->active.store(1);
+        m->ctrl->ncons.store(idx + 1);
+        m->chan->consumers.push_back(m);
+    }
     m->upd = std::thread(update_loop, m);
     return VIPER_OK;
 }
@@ -636,7 +763,6 @@ viper_status viper_register_model(const char *model_name, int32_t role, const vi
         m->device = c.device;
         m->cfg = c;
         st = build_manifest(m->man, tensors, n, c.chunk_bytes, c.align, c.device);
-        if (!st) st = alloc_scratch(m);
         if (!st) {
             m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device);
             if (bs && bs->world > 1) {
@@ -700,7 +826,9 @@ viper_status viper_acquire_latest(viper_model *m, uint64_t min_version, int64_t 
                                                   (unsigned long long)min_version);
             if (now >= deadline) return set_error(VIPER_E_TIMEOUT, "acquire timed out");
             const int64_t left_us = (deadline - now) / 1000;
-            futex_wait(&r->done_seq, seq, std::min<int64_t>(left_us, 1000));
+            r->waiters.fetch_add(1);
+            if (r->done_seq.load() == seq) futex_wait(&r->done_seq, seq, std::min<int64_t>(left_us, 1000));
+            r->waiters.fetch_sub(1);
             continue;
         }
         const int slot = (int)(s & 1);
@@ -770,7 +898,9 @@ viper_status viper_wait_installed(viper_model *m, uint64_t v, int64_t timeout_us
         if (r->done_version.load() >= v && r->last_status.load() != VIPER_OK) return r->last_status.load();
         const int64_t now = now_ns();
         if (now >= deadline) return set_error(VIPER_E_TIMEOUT, "version %llu not installed in time", (unsigned long long)v);
-        futex_wait(&r->done_seq, seq, std::min<int64_t>((deadline - now) / 1000, 1000));
+        r->waiters.fetch_add(1);
+        if (r->done_seq.load() == seq) futex_wait(&r->done_seq, seq, std::min<int64_t>((deadline - now) / 1000, 1000));
+        r->waiters.fetch_sub(1);
     }
 }
 
@@ -780,7 +910,8 @@ viper_status viper_get_stats(viper_model *m, viper_stats *out) {
         float ms = 0;
         if (cudaEventElapsedTime(&ms, m->ev_t[0], m->ev_t[1]) == cudaSuccess) {
             std::lock_guard<std::mutex> lk(m->stats_mu);
-            m->stats.t_pack_dev_us = ms * 1e3;
+            if (m->last_fused) m->stats.t_fused_dev_us = ms * 1e3;
+            else m->stats.t_pack_dev_us = ms * 1e3;
         }
         m->timing_pending = false;
     }
@@ -805,12 +936,18 @@ viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_s
     if (nchunks) *nchunks = m->man.nchunks;
     if (m->role == VIPER_PRODUCER) {
         const int b = m->cur_snap;
+        if (m->ev_sealed[b]) CUDA_TRY(cudaEventSynchronize(m->ev_sealed[b]));
         if (dev_packed) *dev_packed = m->d_snap[b];
         if (dev_seals) *dev_seals = m->d_seal[b];
     } else {
         if (dev_packed) *dev_packed = m->d_stage;
-        if (dev_seals) *dev_seals = m->d_stage_seals;
+        if (dev_seals) *dev_seals = nullptr;
     }
+    return VIPER_OK;
+}
+
+viper_status viper_debug_trace(int64_t *out, int32_t n) {
+    for (int i = 0; i < n && i < 16; i++) out[i] = g_trace[i];
     return VIPER_OK;
 }
 

@@ -36,6 +36,7 @@ struct alignas(64) ConsRec {
     std::atomic<int64_t> ref[2];         // readers pinning each slot
     std::atomic<uint64_t> done_version;  // last version processed (installed or failed)
     std::atomic<uint32_t> done_seq;      // futex word, bumped after each install attempt
+    std::atomic<int32_t> waiters;        // threads sleeping on done_seq
     std::atomic<int32_t> last_status;
     std::atomic<uint64_t> p1_done;       // scatter-allgather: phase-1 version finished
     std::atomic<uint64_t> p2_done;       // scatter-allgather: phase-2 version finished
@@ -51,14 +52,21 @@ struct alignas(64) Ctrl {
     ConsRec cons[kMaxConsumers];
 };
 
+// Pointer-free work item (the device lists add each endpoint's tensor address).
+struct BaseItem {
+    uint64_t tensor_off, packed_off;
+    uint32_t nbytes, chunk, tensor;
+};
+
 struct Manifest {
     int32_t n = 0;
     std::vector<uint64_t> nbytes, offsets;
     uint64_t s_packed = 0, chunk_bytes = 0;
     uint32_t align = 0;
-    std::vector<Item> items;
+    std::vector<BaseItem> items;
+    std::vector<uint32_t> chunk_first;  // [nchunks + 1]
     uint32_t nchunks = 0;
-    Item *d_items = nullptr;
+    uint32_t *d_chunk_first = nullptr;
 };
 
 struct Channel;
@@ -75,8 +83,7 @@ struct viper_model {
     viper_config cfg{};
     vp::Manifest man;
     vp::Geometry geo{};
-    vp::Scratch scratch{};
-    void *scratch_alloc = nullptr;
+    uint32_t *d_flags = nullptr;       // consumer: [0] done blocks, [1] error bits
     vp::Channel *chan = nullptr;       // in-process channel (registry entry)
     vp::Ctrl *ctrl = nullptr;          // host view of the control block
     vp::Ctrl *ctrl_dev = nullptr;      // device view (mapped)
@@ -85,17 +92,20 @@ struct viper_model {
 
     // ---------------- producer
     std::vector<void *> src_ptrs;
-    const uint8_t **d_src = nullptr;
+    vp::Item *d_items = nullptr;                     // producer list / consumer slot-0 list
     uint8_t *d_snap[2] = {nullptr, nullptr};
-    vp::Seal *d_seal[2] = {nullptr, nullptr};
+    vp::ISeal *d_iseal[2] = {nullptr, nullptr};      // item seals + ready flags per snapshot slot
+    vp::Seal *d_seal[2] = {nullptr, nullptr};        // chunk seals per snapshot slot
+    cudaEvent_t ev_sealed[2] = {nullptr, nullptr};   // chunk seals of slot b reduced
     void *snap_alloc = nullptr;
     cudaEvent_t ev_ready[2] = {nullptr, nullptr};   // snapshot slot b complete
     cudaEvent_t ev_packed = nullptr;
     cudaEvent_t ev_t[2] = {nullptr, nullptr};        // VIPER_FLAG_TIMING: around the kernel
     bool timing_pending = false;
+    bool last_fused = false;                         // last publish used publish_fused_kernel
     cudaStream_t side = nullptr;                     // DRAM-tier D2H stream
     uint8_t *h_stage[2] = {nullptr, nullptr};        // DRAM tier (pinned)
-    vp::Seal *h_seal[2] = {nullptr, nullptr};
+    vp::ISeal *h_iseal[2] = {nullptr, nullptr};
     void *h_stage_alloc = nullptr;
     uint64_t snap_version[2] = {0, 0};
     uint64_t last_version = 0;
@@ -105,10 +115,10 @@ struct viper_model {
     int32_t cidx = -1;
     vp::ConsRec *rec = nullptr, *rec_dev = nullptr;
     std::vector<void *> slot_ptrs[2];
-    uint8_t **d_slot[2] = {nullptr, nullptr};
+    vp::Item *d_slot_items[2] = {nullptr, nullptr};  // consumer work lists per slot
     void *slot1_alloc = nullptr;
     uint8_t *d_stage = nullptr;                      // DRAM tier device staging
-    vp::Seal *d_stage_seals = nullptr;
+    vp::ISeal *d_stage_iseal = nullptr;
     void *stage_alloc = nullptr;
     cudaStream_t ustream = nullptr;
     std::thread upd;

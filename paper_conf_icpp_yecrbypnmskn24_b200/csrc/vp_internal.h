@@ -7,15 +7,16 @@
 namespace vp {
 
 // One warp work item: a <= item_max byte piece of one tensor that lies inside
-// one seal chunk.  The same list drives pack (tensor -> packed) and install
-// (packed -> slot tensor): LAY depends only on the sizes, never on pointers.
+// one seal chunk.  `ptr` is the absolute device address of the piece in the
+// tensor (producer: its parameter; consumer: the slot's copy), so a warp needs
+// one dependent load (the item) before it streams data.
 struct Item {
+    uint64_t ptr;          // tensor-side address of this piece
     uint64_t packed_off;   // byte offset in the packed buffer (16-B aligned)
-    uint64_t tensor_off;   // byte offset inside the tensor
     uint32_t nbytes;       // bytes of this piece (multiple of 16 except a tensor tail)
-    uint32_t tensor;       // tensor index
     uint32_t chunk;        // seal chunk index
-    uint32_t chunk_items;  // number of items of that chunk (last-arriver test)
+    uint32_t tensor;       // tensor index
+    uint32_t pad;
 };
 static_assert(sizeof(Item) == 32, "Item must stay 32 B");
 
@@ -24,55 +25,89 @@ struct Seal {
     uint64_t cks;
 };
 
-// Checksum weight constant (R16 / CKS): term_g = w_g * ((2g+1)*K) mod 2^32.
-constexpr uint32_t kCksK = 0x9E3779B1u;
-
-// Per-launch scratch that the kernels leave zeroed when they finish
-// (self-resetting: no memset launch between versions).
-struct Scratch {
-    uint64_t *acc;      // [nchunks] running checksum of the chunk
-    uint32_t *cnt;      // [nchunks] items finished in the chunk
-    uint32_t *done;     // [1] chunks finished
-    uint32_t *err;      // [1] error bits of this launch
+// Item seal: cks(item) + version * kVerMix, then the item's version as a
+// ready flag (written with release semantics after the item's data).
+struct ISeal {
+    uint64_t mixed;
+    uint64_t version;
 };
+static_assert(sizeof(ISeal) == 16, "ISeal must stay 16 B");
 
-enum : uint32_t { kErrChecksum = 1u, kErrVersion = 2u };
+// CKS weight constant (R16): term_g = w_g * ((2g+1)*K) mod 2^32.
+constexpr uint32_t kCksK = 0x9E3779B1u;
+// Item seal = cks(item) + version * kVerMix (mod 2^64): binds every item's
+// checksum to the version, so stale-but-consistent data fails verification.
+constexpr uint64_t kVerMix = 0x9E3779B97F4A7C15ull;
+
+enum : uint32_t { kErrChecksum = 1u };
 
 struct PackArgs {
-    const Item *items;
-    uint32_t nitems, nchunks;
-    const uint8_t *const *src;  // [T] producer tensor base pointers (device)
+    const Item *items;          // producer list (ptr = parameter tensor piece)
+    uint32_t nitems;
     uint8_t *packed;            // snapshot buffer
-    Seal *seals;                // [nchunks] written {version, cks}
-    Scratch s;
+    ISeal *iseal;               // [nitems] item seals + ready flags (written)
+    uint64_t version;
+};
+
+struct SealReduceArgs {
+    const uint32_t *chunk_first;  // [nchunks + 1] item ranges of the chunks
+    uint32_t nchunks;
+    const ISeal *iseal;
+    Seal *seals;                  // [nchunks] {version, cks} (written)
     uint64_t version;
 };
 
 struct InstallArgs {
-    const Item *items;
-    uint32_t nitems, nchunks;
-    uint8_t *const *dst;        // [T] target slot tensor base pointers (device)
-    const uint8_t *packed;      // source: snapshot (local or peer-mapped) or staging
-    const Seal *seals;          // expected seals (same origin as packed)
-    Scratch s;
+    const Item *items;          // consumer list of the target slot (ptr = slot tensor piece)
+    uint32_t nitems;
+    const uint8_t *packed;      // source: snapshot (local or peer-mapped) or DRAM staging
+    const ISeal *iseal;         // expected item seals + ready flags (same origin as packed)
     uint64_t version;
     uint32_t target;            // slot being written
-    uint32_t fault_item;        // item whose first byte is flipped (fault injection); ~0u = none
-    // Host-mapped control words (cudaHostAlloc/cudaHostRegister mapped).
-    // The last finishing warp writes *status_h, clears *pin_h and, on success,
+    uint32_t fault_item;        // item whose first word is flipped (fault injection); ~0u = none
+    uint32_t *done;             // [1] blocks finished (self-resetting)
+    uint32_t *err;              // [1] error bits (self-resetting)
+    // Host-mapped control words (cudaHostAlloc/cudaHostRegister mapped).  The
+    // last block writes *status_h, clears *pin_h and, when every item matched,
     // flips *state_h = (version << 1) | target: the atomic version swap.
     volatile int32_t *status_h;
     volatile uint64_t *pin_h;
     volatile uint64_t *state_h;
 };
 
-// Work-list geometry chosen on the host (kernels.cu).
+// SYNC in-process publish (K2+K6 fused): each warp packs its item,
+// then reads that snapshot piece back (L2) and installs + verifies it into up
+// to kMaxFused consumers' inactive slots; the last block swaps their versions.
+constexpr int kMaxFused = 4;
+struct FusedCons {
+    const Item *items;          // consumer list of its target slot
+    uint32_t target;
+    uint32_t fault_item;
+    volatile int32_t *status_h;
+    volatile uint64_t *pin_h;
+    volatile uint64_t *state_h;
+};
+struct FusedArgs {
+    const Item *items;          // producer list
+    uint32_t nitems;
+    uint32_t ncons;
+    uint8_t *packed;
+    ISeal *iseal;
+    uint64_t version;
+    uint32_t *done;             // [1] self-resetting
+    uint32_t *err;              // [1] bit k = consumer k failed, self-resetting
+    FusedCons cons[kMaxFused];
+};
+
 struct Geometry {
     int grid, block;
 };
 Geometry pick_geometry(uint32_t nitems, int device);
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
-cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st);
+cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
+cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
+// pdl: the install directly follows the pack on `st` (programmatic dependent launch)
+cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl);
 
 }  // namespace vp

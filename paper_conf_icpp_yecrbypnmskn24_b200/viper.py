@@ -20,6 +20,7 @@ TIER_GPU, TIER_DRAM = 0, 1
 FANOUT_DIRECT, FANOUT_SCATTER_ALLGATHER = 0, 2
 SYNC, ASYNC = 0, 1
 FLAG_TIMING = 2
+FLAG_NO_FUSE = 4
 SCHED_FIXED, SCHED_GREEDY = 0, 1
 
 
@@ -52,7 +53,7 @@ class viper_stats(C.Structure):
                 ("installs", C.c_uint64), ("skipped", C.c_uint64), ("failures", C.c_uint64),
                 ("t_publish_us", C.c_double), ("t_install_us", C.c_double), ("t_notify_us", C.c_double),
                 ("writer_wait_us", C.c_double), ("t_pack_dev_us", C.c_double),
-                ("t_install_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32)]
+                ("t_install_dev_us", C.c_double), ("t_fused_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32)]
 
 
 class viper_sched_in(C.Structure):

@@ -19,6 +19,8 @@ def lib():
         _lib.vgen_fill.restype = C.c_int
         _lib.l2_flush.argtypes = [C.c_void_p, C.c_uint64, C.c_void_p]
         _lib.l2_flush.restype = C.c_int
+        _lib.launch_empty.argtypes = [C.c_void_p]
+        _lib.launch_empty.restype = C.c_int
     return _lib
 
 
@@ -50,3 +52,8 @@ def alloc_model(specs, device="cuda:0"):
 def l2_flush(buf, stream=None):
     if lib().l2_flush(C.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(), _sp(stream)) != 0:
         raise RuntimeError("l2_flush failed")
+
+
+def empty_kernel(stream=None):
+    if lib().launch_empty(_sp(stream)) != 0:
+        raise RuntimeError("launch_empty failed")

@@ -77,12 +77,13 @@ def close_all(prod, cons):
 
 
 # ------------------------------------------------------------------ C1 (BJ configs[0])
-@pytest.mark.parametrize("tier", [V.TIER_GPU, V.TIER_DRAM])
-@pytest.mark.parametrize("mode", [V.SYNC, V.ASYNC])
-def test_c1_ptychonn_10_versions(tier, mode):
+@pytest.mark.parametrize("tier,mode,flags", [(V.TIER_GPU, V.SYNC, 0), (V.TIER_GPU, V.SYNC, V.FLAG_NO_FUSE),
+                                              (V.TIER_GPU, V.ASYNC, 0), (V.TIER_DRAM, V.SYNC, 0),
+                                              (V.TIER_DRAM, V.ASYNC, 0)])
+def test_c1_ptychonn_10_versions(tier, mode, flags):
     specs = synth.model_specs("ptychonn")
     seed = synth.SEEDS["ptychonn"]
-    prod, prod_t, cons, cons_t = make_pair(specs, seed, tier=tier, mode=mode)
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, tier=tier, mode=mode, flags=flags)
     try:
         for v in range(1, 11):
             G.fill_model(prod_t, specs, seed, v)
@@ -117,7 +118,9 @@ def test_ragged_tensor_lists_many_chunks(seed):
         specs.append((f"t{i}", dt, (ne,)))
     chunk = int(rng.choice([256, 4096, 65536]))
     align = int(rng.choice([16, 256]))
-    prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=3, chunk_bytes=chunk, align=align)
+    flags = V.FLAG_NO_FUSE if seed % 2 else 0
+    ncons = 3 if seed < 4 else 6   # > kMaxFused local consumers -> separate kernels
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=ncons, chunk_bytes=chunk, align=align, flags=flags)
     try:
         for v in (1, 2, 5):
             G.fill_model(prod_t, specs, 77 + seed, v)
@@ -174,10 +177,11 @@ def test_empty_model():
 
 
 # ---------------------------------------------------------------- protocol on device
-def test_fault_injection_keeps_old_version():
+@pytest.mark.parametrize("flags", [0, V.FLAG_NO_FUSE])
+def test_fault_injection_keeps_old_version(flags):
     specs = synth.model_specs("ptychonn")
     seed = 11
-    prod, prod_t, cons, cons_t = make_pair(specs, seed)
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, flags=flags)
     try:
         G.fill_model(prod_t, specs, seed, 1)
         prod.publish(1)

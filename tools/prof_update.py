@@ -1,0 +1,34 @@
+"""Run a few SYNC model updates of one config (for ncu captures; no timing)."""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch
+
+import synth
+from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+from synth import gpu as G
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="ptychonn")
+ap.add_argument("--steps", type=int, default=5)
+ap.add_argument("--flush", action="store_true")
+ap.add_argument("--tier", type=int, default=0)
+a = ap.parse_args()
+specs = synth.model_specs(a.config)
+seed = synth.SEEDS[a.config]
+pt, ct = G.alloc_model(specs), G.alloc_model(specs)
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if a.flush else None
+c = V.Model("prof", V.CONSUMER, ct, tier=a.tier)
+p = V.Model("prof", V.PRODUCER, pt, tier=a.tier)
+for v in range(1, a.steps + 1):
+    G.fill_model(pt, specs, seed, v)
+    if flush is not None:
+        G.l2_flush(flush)
+    p.publish(v)
+torch.cuda.synchronize()
+c.close()
+p.close()
+print("done", a.config, a.steps)
