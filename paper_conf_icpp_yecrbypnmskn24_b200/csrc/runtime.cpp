@@ -70,7 +70,7 @@ static inline void cpu_relax() { __builtin_ia32_pause(); }
 // ------------------------------------------------------------------ manifest
 // LAY (R16) + the warp work list.  Items never cross a seal chunk
 // and are at most item_max bytes; splits fall on 16-B multiples of the tensor.
-static viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes,
+viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes,
                                    uint32_t align, int device) {
     m.n = n;
     m.nbytes.resize(n);
@@ -121,7 +121,7 @@ static viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n
 
 // Device work list of one endpoint: the base items with that endpoint's tensor
 // addresses folded in.
-static viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out) {
+viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out) {
     *d_out = nullptr;
     if (m.items.empty()) return VIPER_OK;
     std::vector<Item> v(m.items.size());
@@ -174,7 +174,7 @@ static void channel_close(Channel *ch) {
 }
 
 // --------------------------------------------------------------- install path
-static void fire_callback(viper_model *c, uint64_t v, viper_status st) {
+void fire_callback(viper_model *c, uint64_t v, viper_status st) {
     void (*cb)(uint64_t, viper_status, void *);
     void *user;
     {
@@ -188,7 +188,7 @@ static void fire_callback(viper_model *c, uint64_t v, viper_status st) {
 // Pin the latest published snapshot (Dekker pair with the producer's
 // pub_state store -> pin scan).  Returns false when
 // nothing is published.
-static bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
+bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
     for (;;) {
         const uint64_t ps = ctrl->pub_state.load();
         if (ps == 0) return false;
@@ -202,16 +202,10 @@ static bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
     }
 }
 
-struct PreparedInstall {
-    viper_model *c = nullptr;
-    InstallArgs a{};
-    double waited_us = 0;
-};
-
 // Host half of an install of snapshot slot b (version v) of producer p into
 // the inactive slot of consumer c: wait until no reader pins the target (a7)
 // and build the kernel arguments.  Caller holds c->install_mu.
-static viper_status prepare_install(viper_model *c, viper_model *p, uint64_t v, int b, PreparedInstall *pi) {
+viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, int b, PreparedInstall *pi) {
     ConsRec *r = c->rec;
     const uint64_t cur = r->state.load();
     const int target = cur == 0 ? 0 : (int)(1 - (cur & 1));
@@ -228,8 +222,8 @@ static viper_status prepare_install(viper_model *c, viper_model *p, uint64_t v, 
     const bool dram = c->cfg.tier == VIPER_TIER_DRAM;
     a.items = c->d_slot_items[target];
     a.nitems = (uint32_t)c->man.items.size();
-    a.packed = dram ? c->d_stage : p->d_snap[b];
-    a.iseal = dram ? c->d_stage_iseal : p->d_iseal[b];
+    a.packed = dram ? c->d_stage : src.snap[b];
+    a.iseal = dram ? c->d_stage_iseal : src.iseal[b];
     a.version = v;
     a.target = (uint32_t)target;
     a.fault_item = ~0u;
@@ -245,14 +239,14 @@ static viper_status prepare_install(viper_model *c, viper_model *p, uint64_t v, 
 // Stream half: [wait for the snapshot] [DRAM tier: H2D staging] install kernel.
 // pdl: the kernel directly follows the pack on st and consumes its items as
 // they are sealed (kernels.cu, item-granular pipeline).
-static viper_status launch_prepared(PreparedInstall &pi, viper_model *p, int b, cudaStream_t st, bool wait_ready,
-                                    bool pdl) {
+viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, cudaStream_t st,
+                                    bool wait_ready, bool pdl) {
     viper_model *c = pi.c;
-    if (wait_ready) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
+    if (wait_ready && src.ev_ready[b]) CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
     if (c->cfg.tier == VIPER_TIER_DRAM) {
         // Host-to-Host channel: host staging -> this GPU's staging
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage, p->h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, p->h_iseal[b], sizeof(ISeal) * c->man.items.size(),
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, src.h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.h_iseal[b], sizeof(ISeal) * c->man.items.size(),
                                  cudaMemcpyHostToDevice, st));
         pdl = false;
     }
@@ -269,16 +263,29 @@ static viper_status launch_prepared(PreparedInstall &pi, viper_model *p, int b, 
     return VIPER_OK;
 }
 
-static viper_status enqueue_install(viper_model *c, viper_model *p, uint64_t v, int b, cudaStream_t st,
+viper_status enqueue_install(viper_model *c, const SnapSource &src, uint64_t v, int b, cudaStream_t st,
                                     bool wait_ready) {
     PreparedInstall pi;
-    viper_status s = prepare_install(c, p, v, b, &pi);
+    viper_status s = prepare_install(c, src, v, b, &pi);
     if (s) return s;
-    return launch_prepared(pi, p, b, st, wait_ready, false);
+    return launch_prepared(pi, src, b, st, wait_ready, false);
+}
+
+// In-process source: the producer's own buffers.
+SnapSource source_of(const viper_model *p) {
+    SnapSource s;
+    for (int b = 0; b < 2; b++) {
+        s.snap[b] = p->d_snap[b];
+        s.iseal[b] = p->d_iseal[b];
+        s.h_stage[b] = p->h_stage[b];
+        s.h_iseal[b] = p->h_iseal[b];
+        s.ev_ready[b] = p->ev_ready[b];
+    }
+    return s;
 }
 
 // After the install kernel of v completed on the host's view of the stream.
-static viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
+viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
     ConsRec *r = c->rec;
     viper_status st = r->status.load();
     if (st == 1) st = set_error(VIPER_E_CUDA, "install kernel did not report");
@@ -306,7 +313,7 @@ static viper_status finish_install(viper_model *c, uint64_t v, double t_install_
     return st;
 }
 
-static void update_loop(viper_model *c) {
+void update_loop(viper_model *c) {
     cudaSetDevice(c->device);
     Ctrl *ctrl = c->ctrl;
     ConsRec *r = c->rec;
@@ -318,9 +325,13 @@ static void update_loop(viper_model *c) {
             // SYNC producers install inline; the thread only catches a consumer
             // up that registered after the last publish.
             std::lock_guard<std::mutex> lk(c->install_mu);
-            viper_model *p = c->chan ? c->chan->producer : nullptr;
-            const bool async = p && p->cfg.mode == VIPER_ASYNC;
-            work = p && ps != 0 && (ps >> 1) > c->attempted && (async || c->attempted == 0);
+            if (c->xproc) {  // cross-process: this thread installs every version it sees
+                work = ps != 0 && (ps >> 1) > c->attempted;
+            } else {
+                viper_model *p = c->chan ? c->chan->producer : nullptr;
+                const bool async = p && p->cfg.mode == VIPER_ASYNC;
+                work = p && ps != 0 && (ps >> 1) > c->attempted && (async || c->attempted == 0);
+            }
         }
         if (!work) {
             // short spin (notification latency), then sleep on the futex
@@ -351,9 +362,14 @@ static void update_loop(viper_model *c) {
         c->attempted = v;
         const int64_t tp = ctrl->pub_time_ns.load();
         const int64_t t0 = now_ns();
-        viper_model *p = c->chan ? c->chan->producer : nullptr;
-        viper_status st = p ? enqueue_install(c, p, v, b, c->ustream, true)
-                            : set_error(VIPER_E_STATE, "producer gone");
+        viper_status st;
+        if (c->xproc) {
+            st = xproc_install(c, v, b);
+        } else {
+            viper_model *p = c->chan ? c->chan->producer : nullptr;
+            st = p ? enqueue_install(c, source_of(p), v, b, c->ustream, true)
+                   : set_error(VIPER_E_STATE, "producer gone");
+        }
         if (st == VIPER_OK) {
             cudaError_t e = cudaStreamSynchronize(c->ustream);
             if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
@@ -376,7 +392,7 @@ static void update_loop(viper_model *c) {
 // Wait until consumer c's install of v reported (mapped status word), without
 // a stream synchronisation: the install kernel's last block writes status and
 // then the version word.
-static viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
+viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
     ConsRec *r = c->rec;
     const int64_t t0 = now_ns();
     for (uint32_t spins = 0;; spins++) {
@@ -407,6 +423,15 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         return set_error(VIPER_E_VERSION, "publish(%llu) after %llu: versions strictly increase from 1",
                          (unsigned long long)v, (unsigned long long)p->last_version);
     Ctrl *ctrl = p->ctrl;
+    if (p->xproc && p->last_version) {
+        // ASYNC cross-process: the previous version's notification (a host
+        // function after its pack) must have named it before slot reuse
+        const int64_t w0 = now_ns();
+        while ((ctrl->pub_state.load() >> 1) != p->last_version) {
+            if (now_ns() - w0 > 60ll * 1000000000ll) return set_error(VIPER_E_TIMEOUT, "previous publish stuck");
+            sched_yield();
+        }
+    }
     const int b = p->cur_snap ^ 1;
     const uint64_t old_v = p->snap_version[b];
     // Slot b still holds old_v: wait until no consumer reads it (latest-only
@@ -439,7 +464,8 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     // producer waits for these installs itself, so no snapshot pin is needed.
     std::vector<std::unique_lock<std::mutex>> locks;
     std::vector<PreparedInstall> prepared;
-    if (sync) {
+    const SnapSource psrc = source_of(p);
+    if (sync && p->chan) {
         std::vector<viper_model *> cons;
         {
             std::lock_guard<std::mutex> lk(g_reg_mu);
@@ -449,7 +475,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
             std::unique_lock<std::mutex> lk(c->install_mu);
             if (c->attempted >= v) continue;
             PreparedInstall pi;
-            viper_status s = prepare_install(c, p, v, b, &pi);
+            viper_status s = prepare_install(c, psrc, v, b, &pi);
             if (s != VIPER_OK) {
                 result = s;
                 continue;
@@ -507,7 +533,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     p->last_fused = fuse;
     auto launch_all = [&]() {
         for (PreparedInstall &pi : prepared) {
-            viper_status s = launch_prepared(pi, p, b, st, dram, !dram && launched.empty());
+            viper_status s = launch_prepared(pi, psrc, b, st, dram, !dram && launched.empty());
             if (s != VIPER_OK) {
                 result = s;
                 continue;
@@ -521,8 +547,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     p->snap_version[b] = v;
     p->cur_snap = b;
     p->last_version = v;
-    ctrl->pub_state.store((v << 1) | (uint64_t)b);
-    ctrl->pub_time_ns.store(now_ns());
+    if (!p->xproc) {  // in process, consumers order themselves after ev_ready[b]
+        ctrl->pub_state.store((v << 1) | (uint64_t)b);
+        ctrl->pub_time_ns.store(now_ns());
+    }
     // chunk seals (R16) from the item seals, on the side stream
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
     CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
@@ -545,7 +573,12 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     TRACE(4);
     if (sync && dram) launch_all();
 
-    if (sync) {
+    if (p->xproc) {
+        // remote consumers read slot b without events: name v only once the
+        // snapshot (and, DRAM tier, its host copy) is complete
+        viper_status s = xproc_notify(p, v, b, dram ? p->side : st, sync);
+        if (s != VIPER_OK) result = s;
+    } else if (sync) {
         const int64_t ti = now_ns();
         for (viper_model *c : launched) {
             viper_status s = wait_install_done(c, v, st);
@@ -598,6 +631,7 @@ static void free_model(viper_model *m) {
     cudaSetDevice(m->device);
     cudaDeviceSynchronize();
     if (m->rec) m->rec->active.store(0);
+    if (m->xproc) xproc_free(m);
     if (m->chan) {
         {
             std::lock_guard<std::mutex> lk(g_reg_mu);
@@ -629,7 +663,7 @@ static uint64_t al256(uint64_t x) { return (x + 255) / 256 * 256; }
 
 // Producer-side buffers: two snapshot slots (the latest + the one being
 // filled), their item seals and chunk seals, the events and side stream.
-static viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) {
+viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) {
     const uint64_t S = al256(m->man.s_packed);
     const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
     const uint64_t CS = al256(sizeof(Seal) * std::max<uint32_t>(m->man.nchunks, 1));
@@ -652,7 +686,7 @@ static viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) 
     CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
     CUDA_TRY(cudaMalloc(&m->d_flags, 64));
     CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
-    if (m->cfg.tier == VIPER_TIER_DRAM) {
+    if (m->cfg.tier == VIPER_TIER_DRAM && !m->xproc) {  // cross-process: in the shm segment (xproc.cpp)
         CUDA_TRY(cudaHostAlloc(&m->h_stage_alloc, 2 * (S + IS), cudaHostAllocPortable));
         uint8_t *h = (uint8_t *)m->h_stage_alloc;
         for (int b = 0; b < 2; b++) {
@@ -665,7 +699,7 @@ static viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) 
 
 // Consumer-side buffers: slot 1 (unless supplied), per-slot work lists,
 // completion flags, DRAM-tier staging, the update stream.
-static viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
+viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
     viper_status st;
     const uint64_t S = m->man.s_packed;
     for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[0].push_back(tensors[i].dev_ptr);
@@ -730,8 +764,6 @@ using namespace vp;
 // =================================================================== C-ABI
 extern "C" {
 
-viper_status viper_xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
-viper_status viper_xproc_publish(viper_model *m, uint64_t version, cudaStream_t st);
 
 viper_status viper_register_model(const char *model_name, int32_t role, const viper_tensor *tensors, int32_t n,
                                   const viper_config *cfg, const viper_bootstrap *bs, viper_model **out) {
@@ -767,7 +799,7 @@ viper_status viper_register_model(const char *model_name, int32_t role, const vi
             m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device);
             if (bs && bs->world > 1) {
                 m->xproc = true;
-                st = viper_xproc_register(m, tensors, bs);
+                st = xproc_register(m, tensors, bs);
             } else {
                 st = register_local(m, tensors);
             }
@@ -796,7 +828,6 @@ viper_status viper_publish(viper_model *m, uint64_t version, void *cuda_stream) 
     if (m->role != VIPER_PRODUCER) return set_error(VIPER_E_STATE, "publish on a consumer");
     try {
         if (cudaSetDevice(m->device) != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice");
-        if (m->xproc) return viper_xproc_publish(m, version, (cudaStream_t)cuda_stream);
         return producer_publish(m, version, (cudaStream_t)cuda_stream);
     } catch (const std::exception &e) {
         return set_error(VIPER_E_NOMEM, "publish: %s", e.what());

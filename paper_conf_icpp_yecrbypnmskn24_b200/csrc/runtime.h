@@ -71,6 +71,18 @@ struct Manifest {
 
 struct Channel;
 
+// Where a consumer reads snapshot slot b from: the producer's device buffers
+// (same process, or CUDA-IPC peer-mapped over NVLink), the host staging of the
+// DRAM tier (pinned; a shared-memory segment across processes), and -- in
+// process only -- the event that marks slot b complete.
+struct SnapSource {
+    const uint8_t *snap[2] = {nullptr, nullptr};
+    const ISeal *iseal[2] = {nullptr, nullptr};
+    const uint8_t *h_stage[2] = {nullptr, nullptr};
+    const ISeal *h_iseal[2] = {nullptr, nullptr};
+    cudaEvent_t ev_ready[2] = {nullptr, nullptr};
+};
+
 struct ViewTicket {
     int32_t slot;
 };
@@ -133,6 +145,17 @@ struct viper_model {
     std::unordered_map<uint64_t, vp::ViewTicket> views;
     uint64_t next_ticket = 1;
 
+    // ---------------- cross-process (xproc.cpp)
+    vp::SnapSource xsrc;                             // consumer: peer-mapped producer buffers
+    void *shm_base = nullptr;                        // mapped control segment (+ DRAM staging)
+    size_t shm_bytes = 0;
+    std::string shm_name;
+    bool shm_owner = false;
+    bool shm_registered = false;
+    void *peer_snap_base = nullptr;                  // cudaIpcOpenMemHandle result
+    int32_t nconsumers_x = 0;                        // xproc: consumers in the channel
+    int32_t rank = 0, world = 1;
+
     // ---------------- stats
     std::mutex stats_mu;
     viper_stats stats{};
@@ -149,10 +172,36 @@ struct Channel {
     std::vector<uint64_t> nbytes;  // manifest check
 };
 
+struct PreparedInstall {
+    viper_model *c = nullptr;
+    InstallArgs a{};
+    double waited_us = 0;
+};
+
 // runtime.cpp helpers used by other translation units
 viper_status set_error(viper_status st, const char *fmt, ...);
 int64_t now_ns();
 void futex_wake_all(std::atomic<uint32_t> *w);
 void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us);
+viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes, uint32_t align,
+                            int device);
+viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out);
+bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b);
+viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, int b, PreparedInstall *pi);
+viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, cudaStream_t st, bool wait_ready,
+                             bool pdl);
+viper_status enqueue_install(viper_model *c, const SnapSource &src, uint64_t v, int b, cudaStream_t st,
+                             bool wait_ready);
+viper_status finish_install(viper_model *c, uint64_t v, double t_install_us);
+void update_loop(viper_model *c);
+viper_status alloc_producer(viper_model *m, const viper_tensor *tensors);
+viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors);
+SnapSource source_of(const viper_model *p);
+
+// xproc.cpp
+viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
+viper_status xproc_install(viper_model *c, uint64_t v, int b);   // consumer update thread
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, cudaStream_t st, bool sync);  // producer
+void xproc_free(viper_model *m);
 
 }  // namespace vp

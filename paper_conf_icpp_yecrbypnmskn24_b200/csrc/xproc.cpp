@@ -1,14 +1,322 @@
-// xproc.cpp -- cross-process channel (one process per GPU).  Filled in below
-// the in-process path; until then registration reports VIPER_E_UNSUPPORTED.
+// xproc.cpp -- the cross-process channel: one process per GPU (PAPER.md s4.4
+// "GPU-to-GPU memory and Host-to-Host memory" channels), rebuilt
+// for one NVSwitch node:
+//
+//   bootstrap   two allgathers over the caller's process group (records, then
+//               statuses) -- the only use of a collective on this path;
+//   control     the producer creates a shared-memory segment holding the Ctrl
+//               block (+ the DRAM-tier host staging); every rank maps it and
+//               registers it with CUDA (mapped), so install kernels flip their
+//               consumer's version word from the device;
+//   data        consumers CUDA-IPC-map the producer's snapshot allocation and
+//               their install kernel pulls it over NVLink (peer loads), or
+//               copies it from the shared host staging (DRAM tier);
+//   notify      pub_state + a shared futex, written once slot b is complete
+//               (SYNC: after an event sync; ASYNC: a host function on the
+//               producer's side stream) -- "proactively informing consumers of
+//               model updates".
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <sys/statvfs.h>
+#include <unistd.h>
+
+#include <climits>
+#include <cstring>
+#include <new>
+#include <random>
+
 #include "runtime.h"
 
-using namespace vp;
+namespace vp {
 
-extern "C" viper_status viper_xproc_register(viper_model *m, const viper_tensor *, const viper_bootstrap *) {
-    (void)m;
-    return set_error(VIPER_E_UNSUPPORTED, "cross-process channel not built yet");
+namespace {
+
+constexpr uint32_t kPeerMagic = 0x56495052u;  // "VIPR"
+
+struct PeerRec {
+    uint32_t magic;
+    int32_t role, rank, device, pid, status, tier, fanout;
+    uint64_t s_packed, nitems, nchunks, manifest_hash;
+    uint64_t snap_off[2], iseal_off[2];      // inside the producer's IPC allocation
+    uint64_t shm_bytes, stage_off[2], hiseal_off[2];  // inside the shm segment (DRAM tier)
+    char shm_path[128];                      // "/name" (POSIX shm) or an absolute file path
+    cudaIpcMemHandle_t snap_handle;
+};
+
+uint64_t fnv1a(const void *p, size_t n, uint64_t h = 0xcbf29ce484222325ull) {
+    const uint8_t *b = (const uint8_t *)p;
+    for (size_t i = 0; i < n; i++) h = (h ^ b[i]) * 0x100000001b3ull;
+    return h;
 }
 
-extern "C" viper_status viper_xproc_publish(viper_model *, uint64_t, cudaStream_t) {
-    return set_error(VIPER_E_UNSUPPORTED, "cross-process channel not built yet");
+uint64_t manifest_hash(const Manifest &m) {
+    uint64_t h = fnv1a(m.nbytes.data(), m.nbytes.size() * sizeof(uint64_t));
+    h = fnv1a(&m.align, sizeof m.align, h);
+    return fnv1a(&m.chunk_bytes, sizeof m.chunk_bytes, h);
 }
+
+size_t page_up(size_t x) { return (x + 4095) / 4096 * 4096; }
+
+bool is_posix_shm(const char *path) { return path[0] == '/' && strchr(path + 1, '/') == nullptr; }
+
+// Create the segment: POSIX shm when /dev/shm has room, else a file in /tmp
+// (a MAP_SHARED file mapping is shared the same way).
+viper_status create_segment(viper_model *m, size_t bytes, char *path_out, size_t cap) {
+    std::random_device rd;
+    std::string base;
+    for (char ch : m->name) base += (isalnum((unsigned char)ch) ? ch : '_');
+    if (base.size() > 40) base.resize(40);
+    char tag[64];
+    snprintf(tag, sizeof tag, "viper-%s-%d-%08x", base.c_str(), (int)getpid(), (unsigned)rd());
+    struct statvfs sv;
+    const bool shm_ok = statvfs("/dev/shm", &sv) == 0 && (uint64_t)sv.f_bavail * sv.f_frsize > bytes + (64u << 20);
+    int fd;
+    if (shm_ok) {
+        snprintf(path_out, cap, "/%s", tag);
+        fd = shm_open(path_out, O_CREAT | O_EXCL | O_RDWR, 0600);
+    } else {
+        snprintf(path_out, cap, "/tmp/%s", tag);
+        fd = open(path_out, O_CREAT | O_EXCL | O_RDWR, 0600);
+    }
+    if (fd < 0) return set_error(VIPER_E_NOMEM, "cannot create control segment %s", path_out);
+    if (ftruncate(fd, (off_t)bytes) != 0) {
+        close(fd);
+        return set_error(VIPER_E_NOMEM, "ftruncate(%s, %zu) failed", path_out, bytes);
+    }
+    void *p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    close(fd);
+    if (p == MAP_FAILED) return set_error(VIPER_E_NOMEM, "mmap(%s) failed", path_out);
+    m->shm_base = p;
+    m->shm_bytes = bytes;
+    m->shm_name = path_out;
+    m->shm_owner = true;
+    return VIPER_OK;
+}
+
+viper_status open_segment(viper_model *m, const char *path, size_t bytes) {
+    const int fd = is_posix_shm(path) ? shm_open(path, O_RDWR, 0600) : open(path, O_RDWR);
+    if (fd < 0) return set_error(VIPER_E_PEER, "cannot open control segment %s", path);
+    void *p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    close(fd);
+    if (p == MAP_FAILED) return set_error(VIPER_E_PEER, "mmap(%s) failed", path);
+    m->shm_base = p;
+    m->shm_bytes = bytes;
+    m->shm_name = path;
+    return VIPER_OK;
+}
+
+#define CUDA_TRY(x)                                                                                          \
+    do {                                                                                                     \
+        cudaError_t e_ = (x);                                                                                \
+        if (e_ != cudaSuccess)                                                                               \
+            return set_error(VIPER_E_CUDA, "%s failed: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+viper_status map_control(viper_model *m) {
+    CUDA_TRY(cudaHostRegister(m->shm_base, m->shm_bytes, cudaHostRegisterPortable | cudaHostRegisterMapped));
+    m->shm_registered = true;
+    void *d = nullptr;
+    CUDA_TRY(cudaHostGetDevicePointer(&d, m->shm_base, 0));
+    m->ctrl = (Ctrl *)m->shm_base;
+    m->ctrl_dev = (Ctrl *)d;
+    return VIPER_OK;
+}
+
+struct NotifyCtx {
+    Ctrl *ctrl;
+    uint64_t word;
+};
+
+void CUDART_CB notify_fn(void *p) {  // host function: no CUDA calls here
+    NotifyCtx *n = (NotifyCtx *)p;
+    n->ctrl->pub_state.store(n->word);
+    n->ctrl->pub_time_ns.store(now_ns());
+    n->ctrl->pub_seq.fetch_add(1);
+    futex_wake_all(&n->ctrl->pub_seq);
+    delete n;
+}
+
+}  // namespace
+
+viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs) {
+    if (!bs->allgather) return set_error(VIPER_E_INVAL, "bootstrap.allgather is NULL");
+    if (bs->rank < 0 || bs->rank >= bs->world || bs->producer_rank < 0 || bs->producer_rank >= bs->world)
+        return set_error(VIPER_E_INVAL, "bad bootstrap ranks");
+    if (bs->world - 1 > kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+    m->rank = bs->rank;
+    m->world = bs->world;
+    m->nconsumers_x = bs->world - 1;
+    const bool producer = m->role == VIPER_PRODUCER;
+    const bool dram = m->cfg.tier == VIPER_TIER_DRAM;
+    PeerRec me{};
+    me.magic = kPeerMagic;
+    me.role = m->role;
+    me.rank = bs->rank;
+    me.device = m->device;
+    me.pid = (int32_t)getpid();
+    me.tier = m->cfg.tier;
+    me.fanout = m->cfg.fanout;
+    me.s_packed = m->man.s_packed;
+    me.nitems = m->man.items.size();
+    me.nchunks = m->man.nchunks;
+    me.manifest_hash = manifest_hash(m->man);
+    viper_status st = VIPER_OK;
+    if (producer != (bs->rank == bs->producer_rank))
+        st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank", bs->rank);
+    const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
+    const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
+    if (st == VIPER_OK && producer) {
+        st = alloc_producer(m, tensors);
+        const size_t ctrl_bytes = page_up(sizeof(Ctrl));
+        const size_t bytes = ctrl_bytes + (dram ? 2 * (S + IS) : 0);
+        if (st == VIPER_OK) st = create_segment(m, bytes, me.shm_path, sizeof me.shm_path);
+        if (st == VIPER_OK) {
+            memset(m->shm_base, 0, ctrl_bytes);
+            Ctrl *c = new (m->shm_base) Ctrl();
+            c->magic = kCtrlMagic;
+            c->ncons.store(bs->world - 1);
+            st = map_control(m);
+        }
+        if (st == VIPER_OK) {
+            me.shm_bytes = bytes;
+            uint8_t *h = (uint8_t *)m->shm_base + ctrl_bytes;
+            for (int b = 0; b < 2; b++) {
+                me.snap_off[b] = (uint64_t)(m->d_snap[b] - (uint8_t *)m->snap_alloc);
+                me.iseal_off[b] = (uint64_t)((uint8_t *)m->d_iseal[b] - (uint8_t *)m->snap_alloc);
+                if (dram) {
+                    me.stage_off[b] = ctrl_bytes + b * S;
+                    me.hiseal_off[b] = ctrl_bytes + 2 * S + b * IS;
+                    m->h_stage[b] = h + b * S;
+                    m->h_iseal[b] = (ISeal *)(h + 2 * S + b * IS);
+                }
+            }
+            const cudaError_t e = cudaIpcGetMemHandle(&me.snap_handle, m->snap_alloc);
+            if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
+        }
+    }
+    me.status = st;
+    // ---- allgather #1: every rank's record
+    std::vector<PeerRec> all(bs->world);
+    if (bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user) != 0)
+        return set_error(VIPER_E_PEER, "bootstrap allgather failed");
+    const PeerRec &pr = all[bs->producer_rank];
+    if (st == VIPER_OK) {
+        for (int r = 0; r < bs->world; r++) {
+            if (all[r].magic != kPeerMagic) st = set_error(VIPER_E_PEER, "rank %d sent a bad record", r);
+            else if (all[r].status != VIPER_OK) st = set_error(VIPER_E_PEER, "rank %d failed to register", r);
+            else if (all[r].manifest_hash != me.manifest_hash)
+                st = set_error(VIPER_E_INVAL, "rank %d registered a different tensor list", r);
+            else if (all[r].tier != me.tier || all[r].fanout != me.fanout)
+                st = set_error(VIPER_E_INVAL, "rank %d uses another tier / fan-out", r);
+        }
+    }
+    if (st == VIPER_OK && !producer) {
+        int idx = 0;
+        for (int r = 0; r < bs->rank; r++)
+            if (r != bs->producer_rank) idx++;
+        m->cidx = idx;
+        st = open_segment(m, pr.shm_path, pr.shm_bytes);
+        if (st == VIPER_OK) st = map_control(m);
+        if (st == VIPER_OK && m->ctrl->magic != kCtrlMagic) st = set_error(VIPER_E_PEER, "bad control segment");
+        if (st == VIPER_OK) {
+            m->rec = &m->ctrl->cons[idx];
+            m->rec_dev = &m->ctrl_dev->cons[idx];
+            const cudaError_t e =
+                cudaIpcOpenMemHandle(&m->peer_snap_base, pr.snap_handle, cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess)
+                st = set_error(VIPER_E_PEER, "cudaIpcOpenMemHandle (producer rank %d): %s", bs->producer_rank,
+                               cudaGetErrorString(e));
+        }
+        if (st == VIPER_OK) {
+            for (int b = 0; b < 2; b++) {
+                m->xsrc.snap[b] = (const uint8_t *)m->peer_snap_base + pr.snap_off[b];
+                m->xsrc.iseal[b] = (const ISeal *)((const uint8_t *)m->peer_snap_base + pr.iseal_off[b]);
+                if (dram) {
+                    m->xsrc.h_stage[b] = (const uint8_t *)m->shm_base + pr.stage_off[b];
+                    m->xsrc.h_iseal[b] = (const ISeal *)((const uint8_t *)m->shm_base + pr.hiseal_off[b]);
+                }
+            }
+            st = alloc_consumer(m, tensors);
+        }
+        if (st == VIPER_OK) m->rec->active.store(1);
+    }
+    // ---- allgather #2: statuses (all ranks fail together)
+    PeerRec fin{};
+    fin.magic = kPeerMagic;
+    fin.status = st;
+    std::vector<PeerRec> sts(bs->world);
+    if (bs->allgather(&fin, sts.data(), sizeof(PeerRec), bs->user) != 0)
+        return set_error(VIPER_E_PEER, "bootstrap allgather #2 failed");
+    if (st != VIPER_OK) return st;
+    for (int r = 0; r < bs->world; r++)
+        if (sts[r].status != VIPER_OK) return set_error(VIPER_E_PEER, "rank %d failed to register", r);
+    if (!producer) m->upd = std::thread(update_loop, m);
+    return VIPER_OK;
+}
+
+// Consumer update thread (install_mu held, v pinned): pull slot b of the
+// producer over the peer mapping (or from the shared DRAM staging).
+viper_status xproc_install(viper_model *c, uint64_t v, int b) {
+    return enqueue_install(c, c->xsrc, v, b, c->ustream, false);
+}
+
+// Producer: name v in pub_state once slot b is complete on `ready_st`.
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, cudaStream_t ready_st, bool sync) {
+    Ctrl *ctrl = p->ctrl;
+    const uint64_t word = (v << 1) | (uint64_t)b;
+    if (!sync) {
+        // after the seal reduction (and the D2H) on the side stream: the
+        // caller's stream is never blocked by the notification
+        NotifyCtx *n = new NotifyCtx{ctrl, word};
+        const cudaError_t e = cudaLaunchHostFunc(p->side, notify_fn, n);
+        if (e != cudaSuccess) {
+            delete n;
+            return set_error(VIPER_E_CUDA, "cudaLaunchHostFunc: %s", cudaGetErrorString(e));
+        }
+        (void)ready_st;
+        return VIPER_OK;
+    }
+    CUDA_TRY(cudaEventSynchronize(p->ev_ready[b]));
+    ctrl->pub_state.store(word);
+    ctrl->pub_time_ns.store(now_ns());
+    ctrl->pub_seq.fetch_add(1);
+    futex_wake_all(&ctrl->pub_seq);
+    // SYNC: every active consumer processed v (installed or failed)
+    viper_status worst = VIPER_OK;
+    const int nc = ctrl->ncons.load();
+    for (int i = 0; i < nc; i++) {
+        ConsRec *r = &ctrl->cons[i];
+        const int64_t t0 = now_ns();
+        for (;;) {
+            const uint32_t seq = r->done_seq.load();
+            if (!r->active.load() || r->done_version.load() >= v) break;
+            if (now_ns() - t0 > 60ll * 1000000000ll)
+                return set_error(VIPER_E_TIMEOUT, "consumer %d did not install v%llu", i, (unsigned long long)v);
+            r->waiters.fetch_add(1);
+            if (r->done_seq.load() == seq && r->done_version.load() < v) futex_wait(&r->done_seq, seq, 1000);
+            r->waiters.fetch_sub(1);
+        }
+        if (r->active.load() && r->done_version.load() == v && r->last_status.load() != VIPER_OK && worst == VIPER_OK)
+            worst = set_error(r->last_status.load(), "consumer %d failed to install v%llu", i, (unsigned long long)v);
+    }
+    return worst;
+}
+
+void xproc_free(viper_model *m) {
+    if (m->role == VIPER_PRODUCER && m->ctrl) m->ctrl->closing.store(1);
+    if (m->peer_snap_base) cudaIpcCloseMemHandle(m->peer_snap_base);
+    m->peer_snap_base = nullptr;
+    if (m->shm_registered) cudaHostUnregister(m->shm_base);
+    m->shm_registered = false;
+    if (m->shm_base) munmap(m->shm_base, m->shm_bytes);
+    m->shm_base = nullptr;
+    m->ctrl = nullptr;
+    m->rec = nullptr;
+    if (m->shm_owner) {
+        if (is_posix_shm(m->shm_name.c_str())) shm_unlink(m->shm_name.c_str());
+        else unlink(m->shm_name.c_str());
+    }
+}
+
+}  // namespace vp

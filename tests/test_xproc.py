@@ -1,0 +1,49 @@
+"""Cross-process channel (one process per GPU).  The GPU cases run the worker
+under torchrun with every rank on cuda:0 (CUDA-IPC to the same device): the
+same registration / peer-mapping / notification / install code that spans
+GPUs on an 8-GPU box.  The CPU case checks the bootstrap allgather marshalling
+over a world-size-2 gloo group."""
+import os
+import socket
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def run_torchrun(nproc, script, args, timeout=240):
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), script] + args
+    r = subprocess.run(cmd, cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, timeout=timeout, text=True)
+    return r.returncode, r.stdout
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,tier,mode,config", [
+    (2, 0, 0, "ptychonn"), (4, 0, 0, "small"), (3, 0, 1, "small"), (2, 1, 0, "small"), (3, 1, 1, "ptychonn"),
+])
+def test_xproc_parity(nproc, tier, mode, config):
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", config, "--tier", str(tier), "--mode", str(mode)])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+def test_xproc_fault_injection():
+    rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fault", "1", "--versions", "3"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+def test_bootstrap_allgather_gloo_world2():
+    rc, out = run_torchrun(2, "tests/bootstrap_worker.py", [], timeout=120)
+    assert rc == 0 and "BOOTSTRAP_OK" in out, out[-3000:]

@@ -1,0 +1,120 @@
+"""Worker for the cross-process tests (one process per "GPU"; on a 1-GPU box
+every rank uses cuda:0 and CUDA-IPC maps the same device).
+
+Rank 0 = producer, ranks 1.. = consumers; bootstrap over a gloo group.
+Checks, for every version: each consumer's acquired view is byte-identical to
+VGEN(version) computed on the host (synth.vgen_numpy), versions never go
+backwards, and the producer's chunk seals equal the oracle's.
+"""
+import argparse
+import os
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+import synth
+from oracle import transfer as T
+from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+from synth import gpu as G
+
+
+def host_bytes(t):
+    return t.contiguous().view(torch.uint8).reshape(-1).cpu().numpy() if t.numel() else np.zeros(0, np.uint8)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="ptychonn")
+    ap.add_argument("--tier", type=int, default=0)
+    ap.add_argument("--mode", type=int, default=0)
+    ap.add_argument("--fanout", type=int, default=0)
+    ap.add_argument("--versions", type=int, default=6)
+    ap.add_argument("--fault", type=int, default=0)
+    a = ap.parse_args()
+    dist.init_process_group("gloo")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    dev = rank % torch.cuda.device_count()
+    torch.cuda.set_device(dev)
+    specs = synth.model_specs(a.config) if a.config in synth.SEEDS else \
+        [(f"t{i}", synth.F32, (1000 + 37 * i,)) for i in range(7)] + [("odd", synth.BYTES, (13,))]
+    seed = synth.SEEDS.get(a.config, 0xC0FFEE)
+    tensors = G.alloc_model(specs, device=f"cuda:{dev}")
+    bs = V.Bootstrap(rank, world, producer_rank=0)
+    role = V.PRODUCER if rank == 0 else V.CONSUMER
+    m = V.Model(f"xp-{a.config}", role, tensors, tier=a.tier, mode=a.mode, fanout=a.fanout, device=dev,
+                bootstrap=bs)
+    errors = 0
+    last = 0
+    for v in range(1, a.versions + 1):
+        if a.fault and rank == 1 and v == 2:
+            m.fault_next()
+        dist.barrier()
+        if rank == 0:
+            G.fill_model(tensors, specs, seed, v)
+            torch.cuda.synchronize()
+            try:
+                m.publish(v)
+            except V.ViperError as e:
+                if not (a.fault and v == 2 and e.status == V.E_CHECKSUM):
+                    print(f"[rank0] publish({v}) failed: {e}", flush=True)
+                    errors += 1
+            if a.mode == V.SYNC:
+                _, sp, n = m.debug_buffers()
+                like = torch.empty(4 * n, dtype=torch.int32, device=f"cuda:{dev}")
+                seals = V._from_ptr(sp, like).view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2)
+                exp = [synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
+                off, S = T.layout([e.size for e in exp], 256)
+                if not np.array_equal(seals, T.seal(T.pack(exp, off, S), 2 << 20, v)):
+                    print(f"[rank0] seals differ at v{v}", flush=True)
+                    errors += 1
+        dist.barrier()
+        if rank != 0 and a.mode == V.SYNC:
+            view = m.acquire_latest(timeout_us=5_000_000)
+            want = 1 if (a.fault and rank == 1 and v == 2) else v
+            if view.version != want:
+                print(f"[rank{rank}] v{v}: acquired {view.version}, want {want}", flush=True)
+                errors += 1
+            if view.version < last:
+                errors += 1
+            last = view.version
+            got = view.tensors(tensors)
+            for i, (g, s) in enumerate(zip(got, specs)):
+                if not np.array_equal(host_bytes(g), synth.vgen_numpy(seed, view.version, i, s[1], synth.nelem_of(s))):
+                    print(f"[rank{rank}] tensor {i} differs at v{view.version}", flush=True)
+                    errors += 1
+                    break
+            m.release(view)
+        dist.barrier()
+    if rank != 0 and a.mode == V.ASYNC:
+        m.wait_installed(a.versions, timeout_us=20_000_000)
+        view = m.acquire_latest()
+        if view.version != a.versions:
+            errors += 1
+        got = view.tensors(tensors)
+        for i, (g, s) in enumerate(zip(got, specs)):
+            if not np.array_equal(host_bytes(g), synth.vgen_numpy(seed, view.version, i, s[1], synth.nelem_of(s))):
+                errors += 1
+        m.release(view)
+        st = m.stats()
+        print(f"[rank{rank}] installs={st['installs']} skipped={st['skipped']}", flush=True)
+    dist.barrier()
+    if rank != 0:
+        m.close()
+    dist.barrier()
+    if rank == 0:
+        m.close()
+    t = torch.tensor([errors])
+    dist.all_reduce(t)
+    if rank == 0:
+        print(f"XPROC_RESULT errors={int(t.item())}", flush=True)
+    dist.destroy_process_group()
+    sys.exit(1 if int(t.item()) else 0)
+
+
+if __name__ == "__main__":
+    main()
