@@ -49,6 +49,16 @@ __device__ __forceinline__ void st_release(uint64_t *p, uint64_t v) {
     asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+__device__ __forceinline__ void st_release_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t *p) {
+    uint64_t v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __forceinline__ uint64_t ld_acquire(const uint64_t *p) {
     uint64_t v;
     asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -256,9 +266,37 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
         // with the pack grid (all of whose blocks are resident by then, so
         // this cannot deadlock); wait for item w's ready flag, then stream it
         // with L2-coherent loads.  Without PDL the flag is already set.
+        const uint8_t *src = a.packed + it.packed_off;
+        const ISeal *is = a.iseal + w;
+        uint32_t owner = a.sa_n ? it.chunk % a.sa_n : 0;
+        if (a.sa_n && owner != a.sa_me) {
+            // scatter-allgather: the owner re-publishes this item in its staging
+            int ok = 0;
+            if (lane == 0) {
+                const ISeal *ps = a.sa_isrc[owner] + w;
+                uint32_t backoff = 64;
+                int64_t spent = 0;
+                for (;;) {
+                    if (ld_acquire_sys(&ps->version) == a.version) { ok = 1; break; }
+                    __nanosleep(backoff);
+                    spent += backoff;
+                    if (backoff < 2048) backoff <<= 1;
+                    // the owner is not installing this version (skipped it or
+                    // finished without it): take the item from the producer
+                    if (spent > 20000 && *a.sa_owner_pin[owner] != a.version) break;
+                    if (spent > 50000000) break;  // 50 ms: never hang, fall back
+                }
+            }
+            ok = __shfl_sync(0xffffffffu, ok, 0);
+            if (ok) {
+                src = a.sa_src[owner] + it.packed_off;
+                is = a.sa_isrc[owner] + w;
+            } else {
+                owner = a.sa_me;  // producer copy; not re-published
+            }
+        }
         uint64_t expect = 0;
         if (lane == 0) {
-            const ISeal *is = a.iseal + w;
             uint32_t backoff = 32;
             while (ld_acquire(&is->version) != a.version) {
                 __nanosleep(backoff);
@@ -267,9 +305,38 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             expect = is->mixed;
         }
         __syncwarp();
-        const uint64_t part = warp_sum(copy_item<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes,
-                                                       it.packed_off, lane, w == a.fault_item));
-        if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
+        const bool republish = a.sa_n && owner == a.sa_me && it.chunk % a.sa_n == a.sa_me;
+        if (republish) {
+            // src -> slot, then the slot bytes just stored are read back into
+            // this consumer's staging (what its peers will pull)
+            uint64_t dsts[kMaxFused] = {(uint64_t)(a.sa_stage_out + it.packed_off), 0, 0, 0};
+            uint64_t got[kMaxFused] = {0, 0, 0, 0};
+            const uint64_t part = warp_sum(copy_item_fused(src, (uint8_t *)it.ptr, dsts, 1, it.nbytes, it.packed_off,
+                                                           lane, w == a.fault_item ? 1u : 0u, got));
+            const uint64_t staged = warp_sum(got[0]);
+            __syncwarp();
+            if (lane == 0) {  // peers may now pull item w from this consumer's staging
+                a.sa_iseal_out[w].mixed = expect;
+                st_release_sys(&a.sa_iseal_out[w].version, a.version);
+                if (part + a.version * kVerMix != expect || staged + a.version * kVerMix != expect) bad = true;
+            }
+        } else {
+            uint64_t part = warp_sum(
+                copy_item<true>(src, (uint8_t *)it.ptr, it.nbytes, it.packed_off, lane, w == a.fault_item));
+            const bool from_peer = a.sa_n && owner != a.sa_me;
+            // expect is valid in lane 0 only: take the (warp-uniform) decision there
+            const int heal = __shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0);
+            if (heal) {
+                // a peer's staged copy failed its seal: heal from the producer
+                // (pinned by this consumer) and verify against its own seal
+                const ISeal *ps = a.iseal + w;
+                const uint64_t pexp = lane == 0 ? ps->mixed : 0;
+                part = warp_sum(copy_item<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes,
+                                                it.packed_off, lane, false));
+                if (lane == 0) expect = pexp;
+            }
+            if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
+        }
     }
     if (bad) atomicOr(a.err, kErrChecksum);
     __syncthreads();

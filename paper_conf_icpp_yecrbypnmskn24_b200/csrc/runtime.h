@@ -154,6 +154,10 @@ struct viper_model {
     bool shm_registered = false;
     void *peer_snap_base = nullptr;                  // cudaIpcOpenMemHandle result
     int32_t nconsumers_x = 0;                        // xproc: consumers in the channel
+    void *sa_alloc = nullptr;                        // scatter-allgather: my staging [2][S] + seals [2][n]
+    void *sa_peer_base[vp::kMaxConsumers] = {};          // peers' staging (IPC-opened)
+    void *d_sa_tab = nullptr;                        // device tables: src[2][N], isrc[2][N], pin[N]
+    uint64_t sa_S = 0, sa_IS = 0;
     int32_t rank = 0, world = 1;
 
     // ---------------- stats

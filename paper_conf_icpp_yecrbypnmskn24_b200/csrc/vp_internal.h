@@ -73,6 +73,18 @@ struct InstallArgs {
     volatile int32_t *status_h;
     volatile uint64_t *pin_h;
     volatile uint64_t *state_h;
+    // Scatter-allgather fan-out (sa_n > 0): item x is owned by consumer
+    // chunk(x) % sa_n.  Owned items come from the producer (`packed`) and are
+    // also written to this consumer's staging (+ seal, release.sys) for its
+    // peers; the others are pulled from the owner's staging once its seal
+    // shows `version`, falling back to the producer when the owner is not
+    // installing this version.
+    uint32_t sa_n, sa_me;
+    uint8_t *sa_stage_out;
+    ISeal *sa_iseal_out;
+    const uint8_t *const *sa_src;                // [sa_n] peers' staging (device-mapped)
+    const ISeal *const *sa_isrc;                 // [sa_n] peers' staging seals
+    const volatile uint64_t *const *sa_owner_pin;  // [sa_n] peers' pin words (host-mapped)
 };
 
 // SYNC in-process publish (K2+K6 fused): each warp packs its item,

@@ -42,6 +42,8 @@ struct PeerRec {
     uint64_t shm_bytes, stage_off[2], hiseal_off[2];  // inside the shm segment (DRAM tier)
     char shm_path[128];                      // "/name" (POSIX shm) or an absolute file path
     cudaIpcMemHandle_t snap_handle;
+    cudaIpcMemHandle_t sa_handle;            // consumer staging (scatter-allgather)
+    int32_t cidx;
 };
 
 uint64_t fnv1a(const void *p, size_t n, uint64_t h = 0xcbf29ce484222325ull) {
@@ -137,6 +139,37 @@ void CUDART_CB notify_fn(void *p) {  // host function: no CUDA calls here
     delete n;
 }
 
+viper_status open_sa_peers(viper_model *m, const std::vector<PeerRec> &all, const viper_bootstrap *bs) {
+    const int N = m->nconsumers_x;
+    std::vector<const uint8_t *> src(2 * N), isrc(2 * N);
+    std::vector<const volatile uint64_t *> pins(N);
+    int j = 0;
+    for (int r = 0; r < bs->world; r++) {
+        if (r == bs->producer_rank) continue;
+        uint8_t *base;
+        if (j == m->cidx) {
+            base = (uint8_t *)m->sa_alloc;
+        } else {
+            CUDA_TRY(cudaIpcOpenMemHandle(&m->sa_peer_base[j], all[r].sa_handle, cudaIpcMemLazyEnablePeerAccess));
+            base = (uint8_t *)m->sa_peer_base[j];
+        }
+        for (int b = 0; b < 2; b++) {
+            src[b * N + j] = base + b * m->sa_S;
+            isrc[b * N + j] = base + 2 * m->sa_S + b * m->sa_IS;
+        }
+        pins[j] = (const volatile uint64_t *)&m->ctrl_dev->cons[j].pin;
+        j++;
+    }
+    const size_t bytes = (4 * N + N) * sizeof(void *);
+    CUDA_TRY(cudaMalloc(&m->d_sa_tab, bytes));
+    std::vector<const void *> tab;
+    for (auto p : src) tab.push_back(p);
+    for (auto p : isrc) tab.push_back(p);
+    for (auto p : pins) tab.push_back((const void *)p);
+    CUDA_TRY(cudaMemcpy(m->d_sa_tab, tab.data(), bytes, cudaMemcpyHostToDevice));
+    return VIPER_OK;
+}
+
 }  // namespace
 
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs) {
@@ -195,6 +228,16 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
         }
     }
+    const bool sa = m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER;
+    if (st == VIPER_OK && !producer && sa) {
+        // my staging for the chunks I own, double-buffered by snapshot slot
+        m->sa_S = S;
+        m->sa_IS = IS;
+        cudaError_t e = cudaMalloc(&m->sa_alloc, 2 * (S + IS));
+        if (e == cudaSuccess) e = cudaMemset(m->sa_alloc, 0, 2 * (S + IS));
+        if (e == cudaSuccess) e = cudaIpcGetMemHandle(&me.sa_handle, m->sa_alloc);
+        if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "scatter-allgather staging: %s", cudaGetErrorString(e));
+    }
     me.status = st;
     // ---- allgather #1: every rank's record
     std::vector<PeerRec> all(bs->world);
@@ -239,6 +282,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             }
             st = alloc_consumer(m, tensors);
         }
+        if (st == VIPER_OK && sa) st = open_sa_peers(m, all, bs);
         if (st == VIPER_OK) m->rec->active.store(1);
     }
     // ---- allgather #2: statuses (all ranks fail together)
@@ -258,7 +302,21 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
 // Consumer update thread (install_mu held, v pinned): pull slot b of the
 // producer over the peer mapping (or from the shared DRAM staging).
 viper_status xproc_install(viper_model *c, uint64_t v, int b) {
-    return enqueue_install(c, c->xsrc, v, b, c->ustream, false);
+    if (c->cfg.fanout != VIPER_FANOUT_SCATTER_ALLGATHER || c->nconsumers_x < 2 || c->cfg.tier != VIPER_TIER_GPU)
+        return enqueue_install(c, c->xsrc, v, b, c->ustream, false);
+    PreparedInstall pi;
+    viper_status s = prepare_install(c, c->xsrc, v, b, &pi);
+    if (s) return s;
+    const int N = c->nconsumers_x;
+    const void *const *tab = (const void *const *)c->d_sa_tab;
+    pi.a.sa_n = (uint32_t)N;
+    pi.a.sa_me = (uint32_t)c->cidx;
+    pi.a.sa_stage_out = (uint8_t *)c->sa_alloc + b * c->sa_S;
+    pi.a.sa_iseal_out = (ISeal *)((uint8_t *)c->sa_alloc + 2 * c->sa_S + b * c->sa_IS);
+    pi.a.sa_src = (const uint8_t *const *)(tab + b * N);
+    pi.a.sa_isrc = (const ISeal *const *)(tab + 2 * N + b * N);
+    pi.a.sa_owner_pin = (const volatile uint64_t *const *)(tab + 4 * N);
+    return launch_prepared(pi, c->xsrc, b, c->ustream, false, false);
 }
 
 // Producer: name v in pub_state once slot b is complete on `ready_st`.
@@ -305,6 +363,11 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, cudaStream_t ready_
 
 void xproc_free(viper_model *m) {
     if (m->role == VIPER_PRODUCER && m->ctrl) m->ctrl->closing.store(1);
+    for (auto &p : m->sa_peer_base)
+        if (p) cudaIpcCloseMemHandle(p), p = nullptr;
+    cudaFree(m->d_sa_tab);
+    cudaFree(m->sa_alloc);
+    m->d_sa_tab = m->sa_alloc = nullptr;
     if (m->peer_snap_base) cudaIpcCloseMemHandle(m->peer_snap_base);
     m->peer_snap_base = nullptr;
     if (m->shm_registered) cudaHostUnregister(m->shm_base);

@@ -39,6 +39,22 @@ def test_xproc_parity(nproc, tier, mode, config):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("nproc,mode,config", [(4, 0, "ptychonn"), (3, 0, "small"), (4, 1, "small"),
+                                              (5, 0, "resnet50")])
+def test_xproc_scatter_allgather(nproc, mode, config):
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", config, "--mode", str(mode), "--fanout", "2", "--versions", "5"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+def test_xproc_scatter_allgather_fault():
+    rc, out = run_torchrun(4, "tests/xproc_worker.py", ["--config", "small", "--fanout", "2", "--fault", "1",
+                                                       "--versions", "3"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 def test_xproc_fault_injection():
     rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fault", "1", "--versions", "3"])
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
