@@ -49,6 +49,17 @@ def load_peaks():
         return 6650.0, "fallback"
 
 
+def ncu_traffic(kernel, config):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch from the committed
+    ncu --set full capture (profiles/ncu_traffic.json), or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
+            t = json.load(f)
+        return t.get(f"{kernel}:{config}", {}).get("traffic_bytes")
+    except Exception:
+        return None
+
+
 def dist_env():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
@@ -255,9 +266,129 @@ def cpu_baseline(synth, name, budget_s=10.0, max_updates=400):
             "sample": f"{len(times)} oracle updates of {name} (pack+seal+deliver+verify+install+swap, 1 consumer)"}
 
 
+N_CONFIG = {2: "resnet50", 4: "vit_b16", 8: "gpt2_xl"}  # BASELINE.json configs[1..3]
+
+
+def xproc_arm(args):
+    """N > 1: one process per GPU.  Rank 0 is the producer, ranks 1..N-1 the
+    consumers (1 -> N-1 fan-out over NVLink: direct for one consumer,
+    scatter-allgather for more).  Each step is one SYNC update: rank 0's
+    publish() returns once every consumer swapped.  value = mean update
+    latency (host clock of rank 0 from publish entry to the last consumer's
+    swap); consumers' install-kernel times (CUDA events) are
+    reported as the max over ranks.  An NCCL broadcast of the packed bytes is
+    timed beside it as the baseline."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    from synth import gpu as G
+    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+    rank, world, local = dist_env()
+    ndev = torch.cuda.device_count()
+    dev = local % ndev
+    torch.cuda.set_device(dev)
+    over = ndev < world  # more ranks than GPUs (code-path testing on a 1-GPU box): no NCCL
+    if over:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("cpu:gloo,cuda:nccl", device_id=torch.device("cuda", dev))
+    name = args.config if args.config_explicit else N_CONFIG.get(world, "resnet50")
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    tensors = G.alloc_model(specs)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    gloo = dist.new_group(backend="gloo")
+    bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
+    fanout = V.FANOUT_SCATTER_ALLGATHER if world > 2 else V.FANOUT_DIRECT
+    role = V.PRODUCER if rank == 0 else V.CONSUMER
+    m = V.Model(f"bench-x-{name}", role, tensors, fanout=fanout, flags=V.FLAG_TIMING if rank else 0,
+                device=dev, bootstrap=bs)
+    lat, inst = [], []
+    with ClockSampler(dev) as clk:
+        for i in range(args.warmup + args.steps):
+            v = i + 1
+            if rank == 0:
+                G.fill_model(tensors, specs, seed, v)
+            G.l2_flush(flush)
+            torch.cuda.synchronize()
+            dist.barrier(group=gloo)
+            if rank == 0:
+                t0 = time.perf_counter()
+                m.publish(v)
+                lat.append((time.perf_counter() - t0) * 1e3)
+            dist.barrier(group=gloo)
+            if rank != 0:
+                inst.append(m.stats()["t_install_dev_us"])
+    ok = 1
+    if rank != 0:
+        view = m.acquire_latest()
+        exp = [synth.vgen_bytes_range(seed, view.version, t, s[1], 0, min(4096, synth.nbytes_of(s)))
+               for t, s in enumerate(specs)]
+        got = view.tensors(tensors)
+        import numpy as np
+        for g, e in zip(got, exp):
+            b_ = g.contiguous().view(torch.uint8).reshape(-1)[:e.size].cpu().numpy()
+            ok &= int(np.array_equal(b_, e))
+        ok &= int(view.version == args.warmup + args.steps)
+        m.release(view)
+    # NCCL broadcast baseline of the same bytes (timed on the device, max over ranks)
+    S = synth.model_bytes(name)
+    buf = torch.empty(S, dtype=torch.uint8, device="cuda")
+    nccl_ms = [float("nan")] if over else []
+    for i in range(0 if over else args.warmup + args.steps):
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dist.broadcast(buf, src=0)
+        e1.record()
+        e1.synchronize()
+        if i >= args.warmup:
+            nccl_ms.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.mean(lat[args.warmup:]) if rank == 0 else 0.0,
+                      statistics.median(inst[args.warmup:]) if rank else 0.0,
+                      statistics.mean(nccl_ms), float(1 - ok)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
+    if rank != 0:
+        m.close()
+    dist.barrier(group=gloo)
+    if rank == 0:
+        m.close()
+        peak, peak_kind = load_peaks()
+        lat_ms, inst_us, nccl = float(t[0]), float(t[1]), float(t[2])
+        nvl = 770.0  # measured peer copy GB/s per direction (B200_PROFILING.md)
+        out = {
+            "metric": METRIC, "value": round(lat_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(lat_ms, 6), "higher_is_better": False, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+            "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
+            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers over NVLink "
+                                   f"({'scatter-allgather' if world > 2 else 'direct pull'}), SYNC",
+                       "model_bytes": S, "devices_visible": ndev,
+                       "oversubscribed": ndev < world, "l2": "flushed before every update"},
+            "update_gbps_per_consumer": round(S / (lat_ms * 1e-3) / 1e9, 3),
+            "install_kernel_us_max_over_consumers": round(inst_us, 3),
+            "roofline": None if over else {
+                "bound": "nvlink", "kernel": "install_verify (peer pull)",
+                "achieved": round(S / (inst_us * 1e-6) / 1e9, 2), "peak": nvl, "unit": "GB/s",
+                "frac": round(S / (inst_us * 1e-6) / 1e9 / nvl, 4), "traffic": None,
+                "peak_kind": "measured peer copy (B200_PROFILING.md)"},
+            "nccl_broadcast_ms": None if over else round(nccl, 6),
+            "parity_ok": bool(float(t[3]) == 0.0),
+            "gpu_launches": 3 * args.steps,
+            "clocks": clk.summary(),
+            "e2e": None,
+        }
+        print(json.dumps(out), flush=True)
+    dist.barrier(group=gloo)
+    dist.destroy_process_group()
+
+
 def gpu_arm(args):
     import torch
     rank, world, local = dist_env()
+    if world > 1:
+        return xproc_arm(args)
     torch.cuda.set_device(local)
     import synth
     from synth import gpu as G
@@ -314,7 +445,9 @@ def gpu_arm(args):
                        "how": "library CUDA events around each kernel, stream kept busy (no host gaps); "
                               "event_bracket_floor = an empty kernel timed the same way"},
         "roofline": {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 2), "peak": peak,
-                     "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": None,
+                     "unit": "GB/s", "frac": round(achieved / peak, 4),
+                     "traffic": ncu_traffic("publish_fused_kernel", name),
+                     "traffic_source": "profiles/ncu_traffic.json (ncu --set full, cold caches)",
                      "peak_kind": peak_kind, "algorithmic_bytes": alg},
         "parity_ok": r["ok"],
         "gpu_launches": 2 * args.steps,  # publish_fused + seal_reduce per update
@@ -383,11 +516,14 @@ def main():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="viper", choices=["viper", "reference"])
-    ap.add_argument("--config", default="ptychonn", choices=["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
+    ap.add_argument("--config", default=None, choices=["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    args.config_explicit = args.config is not None
+    if args.config is None:
+        args.config = "ptychonn"
     if args.impl == "reference":
         reference_arm(args)
     else:
