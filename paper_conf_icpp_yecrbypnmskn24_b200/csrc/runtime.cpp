@@ -8,6 +8,7 @@
 // to launch, when, and on which stream.  There is no CPU data path.
 #include "runtime.h"
 
+#include <cuda.h>  // types of the driver entry points (no libcuda link)
 #include <linux/futex.h>
 #include <sched.h>
 #include <sys/syscall.h>
@@ -67,6 +68,36 @@ void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us)
 
 static inline void cpu_relax() { __builtin_ia32_pause(); }
 
+typedef CUresult (*PFN_wait64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+typedef CUresult (*PFN_write64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
+static PFN_wait64 g_wait64 = nullptr;
+static PFN_write64 g_write64 = nullptr;
+static std::once_flag g_memops_once;
+
+static void resolve_memops() {
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuStreamWaitValue64", (void **)&g_wait64, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+        g_wait64 = nullptr;
+    if (cudaGetDriverEntryPoint("cuStreamWriteValue64", (void **)&g_write64, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+        g_write64 = nullptr;
+}
+
+viper_status stream_wait_geq(cudaStream_t st, const void *dev_addr, uint64_t v) {
+    std::call_once(g_memops_once, resolve_memops);
+    if (!g_wait64) return set_error(VIPER_E_UNSUPPORTED, "cuStreamWaitValue64 unavailable");
+    const CUresult r = g_wait64((CUstream)st, (CUdeviceptr)dev_addr, v, CU_STREAM_WAIT_VALUE_GEQ);
+    return r == CUDA_SUCCESS ? VIPER_OK : set_error(VIPER_E_CUDA, "cuStreamWaitValue64 failed (%d)", (int)r);
+}
+
+viper_status stream_write(cudaStream_t st, void *dev_addr, uint64_t v) {
+    std::call_once(g_memops_once, resolve_memops);
+    if (!g_write64) return set_error(VIPER_E_UNSUPPORTED, "cuStreamWriteValue64 unavailable");
+    const CUresult r = g_write64((CUstream)st, (CUdeviceptr)dev_addr, v, CU_STREAM_WRITE_VALUE_DEFAULT);
+    return r == CUDA_SUCCESS ? VIPER_OK : set_error(VIPER_E_CUDA, "cuStreamWriteValue64 failed (%d)", (int)r);
+}
+
 // ------------------------------------------------------------------ manifest
 // LAY (R16) + the warp work list.  Items never cross a seal chunk
 // and are at most item_max bytes; splits fall on 16-B multiples of the tensor.
@@ -113,6 +144,20 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
         m.chunk_first[c + 1] = m.chunk_first[c] + per_chunk[c];
     }
     if (m.items.size() >= (size_t)UINT32_MAX) return set_error(VIPER_E_INVAL, "too many work items");
+    // DRAM-tier pipeline pieces: whole chunks, >= 32 MiB, at most kMaxPieces
+    {
+        const uint64_t want = std::max<uint64_t>(32ull << 20, (m.s_packed + kMaxPieces - 1) / kMaxPieces);
+        const uint64_t per = std::max<uint64_t>(1, (want + chunk_bytes - 1) / chunk_bytes);  // chunks per piece
+        m.piece_lo.clear(); m.piece_hi.clear(); m.piece_ilo.clear(); m.piece_ihi.clear();
+        for (uint64_t c = 0; c < m.nchunks; c += per) {
+            const uint64_t ce = std::min<uint64_t>(m.nchunks, c + per);
+            m.piece_lo.push_back(c * chunk_bytes);
+            m.piece_hi.push_back(std::min<uint64_t>(ce * chunk_bytes, m.s_packed));
+            m.piece_ilo.push_back(m.chunk_first[c]);
+            m.piece_ihi.push_back(m.chunk_first[ce]);
+        }
+        if (m.piece_lo.size() > (size_t)kMaxPieces) return set_error(VIPER_E_INVAL, "too many DRAM pieces");
+    }
     CUDA_TRY(cudaMalloc(&m.d_chunk_first, m.chunk_first.size() * sizeof(uint32_t)));
     CUDA_TRY(cudaMemcpy(m.d_chunk_first, m.chunk_first.data(), m.chunk_first.size() * sizeof(uint32_t),
                         cudaMemcpyHostToDevice));
@@ -242,13 +287,22 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
 viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, cudaStream_t st,
                                     bool wait_ready, bool pdl) {
     viper_model *c = pi.c;
-    if (wait_ready && src.ev_ready[b]) CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
     if (c->cfg.tier == VIPER_TIER_DRAM) {
-        // Host-to-Host channel: host staging -> this GPU's staging
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage, src.h_stage[b], c->man.s_packed, cudaMemcpyHostToDevice, st));
-        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.h_iseal[b], sizeof(ISeal) * c->man.items.size(),
-                                 cudaMemcpyHostToDevice, st));
+        // Host-to-Host channel: host staging -> this GPU's
+        // staging, piece by piece as the producer's D2H lands (GPU-side waits
+        // on the pieces' flags: the D2H and this H2D overlap)
+        const Manifest &mm = c->man;
+        for (size_t i = 0; i < mm.piece_lo.size(); i++) {
+            viper_status s = stream_wait_geq(st, &c->ctrl_dev->dram_flag[b][i], pi.a.version);
+            if (s) return s;
+            CUDA_TRY(cudaMemcpyAsync(c->d_stage + mm.piece_lo[i], src.h_stage[b] + mm.piece_lo[i],
+                                     mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyHostToDevice, st));
+            CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal + mm.piece_ilo[i], src.h_iseal[b] + mm.piece_ilo[i],
+                                     sizeof(ISeal) * (mm.piece_ihi[i] - mm.piece_ilo[i]), cudaMemcpyHostToDevice, st));
+        }
         pdl = false;
+    } else if (wait_ready && src.ev_ready[b]) {
+        CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
     }
     c->rec->status.store(1);  // "in flight"
     const bool timing = c->cfg.flags & VIPER_FLAG_TIMING;
@@ -551,9 +605,33 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         ctrl->pub_state.store((v << 1) | (uint64_t)b);
         ctrl->pub_time_ns.store(now_ns());
     }
-    // chunk seals (R16) from the item seals, on the side stream
+    // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
     CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
+    if (p->xproc && !sync) {
+        // remote consumers read slot b without events: name v once the pack is
+        // complete (host function on the side stream; DRAM-tier consumers
+        // then follow the per-piece flags below)
+        viper_status s = xproc_notify(p, v, b, false);
+        if (s != VIPER_OK) result = s;
+    }
+    if (dram) {
+        // snapshot -> pinned host, piece by piece on the side
+        // stream (the caller's stream is blocked only by the pack); each piece
+        // raises its flag for the consumers' H2D
+        const Manifest &mm = p->man;
+        for (size_t i = 0; i < mm.piece_lo.size(); i++) {
+            CUDA_TRY(cudaMemcpyAsync(p->h_stage[b] + mm.piece_lo[i], p->d_snap[b] + mm.piece_lo[i],
+                                     mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyDeviceToHost, p->side));
+            CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b] + mm.piece_ilo[i], p->d_iseal[b] + mm.piece_ilo[i],
+                                     sizeof(ISeal) * (mm.piece_ihi[i] - mm.piece_ilo[i]), cudaMemcpyDeviceToHost,
+                                     p->side));
+            viper_status s = stream_write(p->side, &p->ctrl_dev->dram_flag[b][i], v);
+            if (s) return s;
+        }
+        CUDA_TRY(cudaEventRecord(p->ev_ready[b], p->side));
+    }
+    // chunk seals (R16) from the item seals
     SealReduceArgs ra{};
     ra.chunk_first = p->man.d_chunk_first;
     ra.nchunks = p->man.nchunks;
@@ -561,23 +639,15 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     ra.seals = p->d_seal[b];
     ra.version = v;
     CUDA_TRY(launch_seal_reduce(ra, p->side));
-    if (dram) {
-        // snapshot -> pinned host on the side stream, so the
-        // caller's stream is blocked only by the pack
-        CUDA_TRY(cudaMemcpyAsync(p->h_stage[b], p->d_snap[b], p->man.s_packed, cudaMemcpyDeviceToHost, p->side));
-        CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b], p->d_iseal[b], sizeof(ISeal) * p->man.items.size(),
-                                 cudaMemcpyDeviceToHost, p->side));
-        CUDA_TRY(cudaEventRecord(p->ev_ready[b], p->side));
-    }
     CUDA_TRY(cudaEventRecord(p->ev_sealed[b], p->side));
     TRACE(4);
     if (sync && dram) launch_all();
 
     if (p->xproc) {
-        // remote consumers read slot b without events: name v only once the
-        // snapshot (and, DRAM tier, its host copy) is complete
-        viper_status s = xproc_notify(p, v, b, dram ? p->side : st, sync);
-        if (s != VIPER_OK) result = s;
+        if (sync) {  // name v once the pack completed, then wait for every consumer
+            viper_status s = xproc_notify(p, v, b, true);
+            if (s != VIPER_OK) result = s;
+        }
     } else if (sync) {
         const int64_t ti = now_ns();
         for (viper_model *c : launched) {

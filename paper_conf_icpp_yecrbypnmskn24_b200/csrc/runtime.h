@@ -26,6 +26,7 @@
 namespace vp {
 
 constexpr int kMaxConsumers = 16;
+constexpr int kMaxPieces = 256;  // DRAM tier: D2H / H2D pipeline granularity (whole chunks)
 constexpr uint64_t kCtrlMagic = 0x5649504552435431ull;  // "VIPERCT1"
 
 struct alignas(64) ConsRec {
@@ -50,6 +51,10 @@ struct alignas(64) Ctrl {
     std::atomic<int64_t> pub_time_ns;    // CLOCK_MONOTONIC of the last publish notification
     std::atomic<int32_t> ncons;
     ConsRec cons[kMaxConsumers];
+    // DRAM tier: piece i of snapshot slot b is in host staging once
+    // dram_flag[b][i] >= v (written by the producer's copy stream with
+    // cuStreamWriteValue64; consumers' copy streams wait with cuStreamWaitValue64)
+    alignas(64) std::atomic<uint64_t> dram_flag[2][kMaxPieces];
 };
 
 // Pointer-free work item (the device lists add each endpoint's tensor address).
@@ -67,6 +72,9 @@ struct Manifest {
     std::vector<uint32_t> chunk_first;  // [nchunks + 1]
     uint32_t nchunks = 0;
     uint32_t *d_chunk_first = nullptr;
+    // DRAM-tier pieces: [byte_lo, byte_hi) and [item_lo, item_hi), whole chunks
+    std::vector<uint64_t> piece_lo, piece_hi;
+    std::vector<uint32_t> piece_ilo, piece_ihi;
 };
 
 struct Channel;
@@ -202,10 +210,14 @@ viper_status alloc_producer(viper_model *m, const viper_tensor *tensors);
 viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors);
 SnapSource source_of(const viper_model *p);
 
+// stream memory operations (driver entry points, resolved at first use)
+viper_status stream_wait_geq(cudaStream_t st, const void *dev_addr, uint64_t v);
+viper_status stream_write(cudaStream_t st, void *dev_addr, uint64_t v);
+
 // xproc.cpp
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
 viper_status xproc_install(viper_model *c, uint64_t v, int b);   // consumer update thread
-viper_status xproc_notify(viper_model *p, uint64_t v, int b, cudaStream_t st, bool sync);  // producer
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync);  // producer, once the pack completed
 void xproc_free(viper_model *m);
 
 }  // namespace vp

@@ -319,23 +319,22 @@ viper_status xproc_install(viper_model *c, uint64_t v, int b) {
     return launch_prepared(pi, c->xsrc, b, c->ustream, false, false);
 }
 
-// Producer: name v in pub_state once slot b is complete on `ready_st`.
-viper_status xproc_notify(viper_model *p, uint64_t v, int b, cudaStream_t ready_st, bool sync) {
+// Producer: name v in pub_state once the pack of slot b completed.  ASYNC:
+// a host function on the side stream (enqueued right after the side stream's
+// wait on the pack).  SYNC: an event sync, then wait for every consumer.
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync) {
     Ctrl *ctrl = p->ctrl;
     const uint64_t word = (v << 1) | (uint64_t)b;
     if (!sync) {
-        // after the seal reduction (and the D2H) on the side stream: the
-        // caller's stream is never blocked by the notification
         NotifyCtx *n = new NotifyCtx{ctrl, word};
         const cudaError_t e = cudaLaunchHostFunc(p->side, notify_fn, n);
         if (e != cudaSuccess) {
             delete n;
             return set_error(VIPER_E_CUDA, "cudaLaunchHostFunc: %s", cudaGetErrorString(e));
         }
-        (void)ready_st;
         return VIPER_OK;
     }
-    CUDA_TRY(cudaEventSynchronize(p->ev_ready[b]));
+    CUDA_TRY(cudaEventSynchronize(p->ev_packed));
     ctrl->pub_state.store(word);
     ctrl->pub_time_ns.store(now_ns());
     ctrl->pub_seq.fetch_add(1);

@@ -1,0 +1,44 @@
+"""DRAM-tier (pinned host staging) update latency vs GPU tier, 1-GPU loopback."""
+import argparse
+import os
+import statistics
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+
+import synth
+from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+from synth import gpu as G
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="resnet50")
+ap.add_argument("--steps", type=int, default=4)
+a = ap.parse_args()
+specs = synth.model_specs(a.config)
+S = synth.model_bytes(a.config)
+pt, ct = G.alloc_model(specs), G.alloc_model(specs)
+for tier in (V.TIER_DRAM, V.TIER_GPU):
+    c = V.Model(f"d{tier}", V.CONSUMER, ct, tier=tier)
+    p = V.Model(f"d{tier}", V.PRODUCER, pt, tier=tier)
+    lat = []
+    for v in range(1, a.steps + 3):
+        G.fill_model(pt, specs, synth.SEEDS[a.config], v)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        p.publish(v)
+        lat.append((time.perf_counter() - t0) * 1e3)
+    lat = lat[2:]
+    print(f"{a.config} tier={'dram' if tier else 'gpu'}: {statistics.mean(lat):.3f} ms/update  "
+          f"({S / (statistics.mean(lat) * 1e-3) / 1e9:.1f} GB/s)", flush=True)
+    c.close()
+    p.close()
+# raw pinned copy rates
+h = torch.empty(S, dtype=torch.uint8).pin_memory()
+d = torch.empty(S, dtype=torch.uint8, device="cuda")
+for name, fn in (("D2H", lambda: h.copy_(d, non_blocking=True)), ("H2D", lambda: d.copy_(h, non_blocking=True))):
+    fn(); torch.cuda.synchronize()
+    t0 = time.perf_counter(); fn(); torch.cuda.synchronize()
+    dt = time.perf_counter() - t0
+    print(f"pinned {name} {S/1e9:.2f} GB: {S / dt / 1e9:.1f} GB/s", flush=True)
