@@ -229,7 +229,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
         __syncwarp();  // every lane's stores are ordered before lane 0's release
         if (lane == 0) {
             a.iseal[w].mixed = part + a.version * kVerMix;
-            st_release(&a.iseal[w].version, a.version);  // item w ready (pipelined install)
+            if (a.sys_release) st_release_sys(&a.iseal[w].version, a.version);  // readers on other GPUs
+            else st_release(&a.iseal[w].version, a.version);  // item w ready (pipelined install)
         }
     }
 }
@@ -295,12 +296,19 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                 owner = a.sa_me;  // producer copy; not re-published
             }
         }
+        // (system scope: the producer may be another GPU pipelining its pack)
         uint64_t expect = 0;
         if (lane == 0) {
             uint32_t backoff = 32;
-            while (ld_acquire(&is->version) != a.version) {
+            uint64_t waited = 0;
+            while (ld_acquire_sys(&is->version) != a.version) {
                 __nanosleep(backoff);
+                waited += backoff;
                 if (backoff < 1024) backoff <<= 1;
+                if (waited > kItemWaitNs) {  // never hang on a vanished producer
+                    atomicOr(a.err, kErrTimeout);
+                    break;
+                }
             }
             expect = is->mixed;
         }
@@ -346,7 +354,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             __threadfence();
             const uint32_t e = atomicExch(a.err, 0u);
             *a.done = 0;
-            const int32_t st = (e & kErrChecksum) ? -5 : 0;
+            const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
             // Every block's slot stores are GPU-visible (cumulative fences
             // above); later readers are kernels launched after the host saw
             // the flip, so plain system-visible stores suffice here.

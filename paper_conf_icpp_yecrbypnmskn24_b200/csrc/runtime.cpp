@@ -577,6 +577,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         a.packed = p->d_snap[b];
         a.iseal = p->d_iseal[b];
         a.version = v;
+        a.sys_release = p->early_notify ? 1u : 0u;
         if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
         CUDA_TRY(launch_pack(a, p->geo, st));
         if (timing) {
@@ -601,14 +602,21 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     p->snap_version[b] = v;
     p->cur_snap = b;
     p->last_version = v;
-    if (!p->xproc) {  // in process, consumers order themselves after ev_ready[b]
+    if (!p->xproc || p->early_notify) {
+        // in process, consumers order themselves after ev_ready[b]; across
+        // GPUs with early notification their install waits per item on the
+        // seals the pack releases at system scope (cross-GPU pipeline)
         ctrl->pub_state.store((v << 1) | (uint64_t)b);
         ctrl->pub_time_ns.store(now_ns());
+        if (p->xproc) {
+            ctrl->pub_seq.fetch_add(1);
+            futex_wake_all(&ctrl->pub_seq);
+        }
     }
     // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
     CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
-    if (p->xproc && !sync) {
+    if (p->xproc && !sync && !p->early_notify) {
         // remote consumers read slot b without events: name v once the pack is
         // complete (host function on the side stream; DRAM-tier consumers
         // then follow the per-piece flags below)
@@ -645,7 +653,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
 
     if (p->xproc) {
         if (sync) {  // name v once the pack completed, then wait for every consumer
-            viper_status s = xproc_notify(p, v, b, true);
+            viper_status s = xproc_notify(p, v, b, true, p->early_notify);
             if (s != VIPER_OK) result = s;
         }
     } else if (sync) {

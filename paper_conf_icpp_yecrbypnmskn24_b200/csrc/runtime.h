@@ -167,6 +167,7 @@ struct viper_model {
     void *d_sa_tab = nullptr;                        // device tables: src[2][N], isrc[2][N], pin[N]
     uint64_t sa_S = 0, sa_IS = 0;
     int32_t rank = 0, world = 1;
+    bool early_notify = false;                       // producer: consumers pipeline behind the pack
 
     // ---------------- stats
     std::mutex stats_mu;
@@ -217,7 +218,7 @@ viper_status stream_write(cudaStream_t st, void *dev_addr, uint64_t v);
 // xproc.cpp
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
 viper_status xproc_install(viper_model *c, uint64_t v, int b);   // consumer update thread
-viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync);  // producer, once the pack completed
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool already = false);  // producer
 void xproc_free(viper_model *m);
 
 }  // namespace vp

@@ -39,7 +39,9 @@ constexpr uint32_t kCksK = 0x9E3779B1u;
 // checksum to the version, so stale-but-consistent data fails verification.
 constexpr uint64_t kVerMix = 0x9E3779B97F4A7C15ull;
 
-enum : uint32_t { kErrChecksum = 1u };
+enum : uint32_t { kErrChecksum = 1u, kErrTimeout = 2u };
+// an install waits at most this long for one item's ready flag (producer gone)
+constexpr uint64_t kItemWaitNs = 30ull * 1000000000ull;
 
 struct PackArgs {
     const Item *items;          // producer list (ptr = parameter tensor piece)
@@ -47,6 +49,8 @@ struct PackArgs {
     uint8_t *packed;            // snapshot buffer
     ISeal *iseal;               // [nitems] item seals + ready flags (written)
     uint64_t version;
+    uint32_t sys_release;       // release the ready flags at system scope (consumers
+                                // on other GPUs pipeline behind this pack)
 };
 
 struct SealReduceArgs {

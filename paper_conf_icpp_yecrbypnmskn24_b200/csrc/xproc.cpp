@@ -44,6 +44,7 @@ struct PeerRec {
     cudaIpcMemHandle_t snap_handle;
     cudaIpcMemHandle_t sa_handle;            // consumer staging (scatter-allgather)
     int32_t cidx;
+    char pci[32];                            // PCI bus id of the rank's GPU
 };
 
 uint64_t fnv1a(const void *p, size_t n, uint64_t h = 0xcbf29ce484222325ull) {
@@ -194,6 +195,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
     me.nitems = m->man.items.size();
     me.nchunks = m->man.nchunks;
     me.manifest_hash = manifest_hash(m->man);
+    cudaDeviceGetPCIBusId(me.pci, sizeof me.pci, m->device);
     viper_status st = VIPER_OK;
     if (producer != (bs->rank == bs->producer_rank))
         st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank", bs->rank);
@@ -253,6 +255,15 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             else if (all[r].tier != me.tier || all[r].fanout != me.fanout)
                 st = set_error(VIPER_E_INVAL, "rank %d uses another tier / fan-out", r);
         }
+    }
+    if (st == VIPER_OK && producer) {
+        // every consumer on another GPU: publish v as soon as the pack is
+        // launched; consumers pull items as their seals are released (.sys)
+        bool other = true;
+        for (int r = 0; r < bs->world; r++)
+            if (r != bs->producer_rank && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
+        const char *env = getenv("VIPER_EARLY_NOTIFY");
+        m->early_notify = env ? atoi(env) != 0 : other;
     }
     if (st == VIPER_OK && !producer) {
         int idx = 0;
@@ -322,7 +333,7 @@ viper_status xproc_install(viper_model *c, uint64_t v, int b) {
 // Producer: name v in pub_state once the pack of slot b completed.  ASYNC:
 // a host function on the side stream (enqueued right after the side stream's
 // wait on the pack).  SYNC: an event sync, then wait for every consumer.
-viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync) {
+viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool already) {
     Ctrl *ctrl = p->ctrl;
     const uint64_t word = (v << 1) | (uint64_t)b;
     if (!sync) {
@@ -334,11 +345,13 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync) {
         }
         return VIPER_OK;
     }
-    CUDA_TRY(cudaEventSynchronize(p->ev_packed));
-    ctrl->pub_state.store(word);
-    ctrl->pub_time_ns.store(now_ns());
-    ctrl->pub_seq.fetch_add(1);
-    futex_wake_all(&ctrl->pub_seq);
+    if (!already) {
+        CUDA_TRY(cudaEventSynchronize(p->ev_packed));
+        ctrl->pub_state.store(word);
+        ctrl->pub_time_ns.store(now_ns());
+        ctrl->pub_seq.fetch_add(1);
+        futex_wake_all(&ctrl->pub_seq);
+    }
     // SYNC: every active consumer processed v (installed or failed)
     viper_status worst = VIPER_OK;
     const int nc = ctrl->ncons.load();

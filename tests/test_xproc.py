@@ -21,10 +21,13 @@ def free_port():
     return p
 
 
-def run_torchrun(nproc, script, args, timeout=240):
+def run_torchrun(nproc, script, args, timeout=240, env=None):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
            "--master-addr", "127.0.0.1", "--master-port", str(free_port()), script] + args
-    r = subprocess.run(cmd, cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, timeout=timeout, text=True)
+    e = dict(os.environ)
+    e.update(env or {})
+    r = subprocess.run(cmd, cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, timeout=timeout, text=True,
+                       env=e)
     return r.returncode, r.stdout
 
 
@@ -51,6 +54,18 @@ def test_xproc_scatter_allgather(nproc, mode, config):
 def test_xproc_scatter_allgather_fault():
     rc, out = run_torchrun(4, "tests/xproc_worker.py", ["--config", "small", "--fanout", "2", "--fault", "1",
                                                        "--versions", "3"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,fanout,mode", [(2, 0, 0), (3, 0, 1), (4, 2, 0)])
+def test_xproc_early_notify_pipeline(nproc, fanout, mode):
+    """Cross-GPU item pipeline: v is published right after the pack launch and
+    consumers' install kernels wait per item on seals released at system scope
+    (forced on here, where all ranks share one GPU)."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", "resnet50", "--fanout", str(fanout), "--mode", str(mode), "--versions", "4"],
+                           env={"VIPER_EARLY_NOTIFY": "1"})
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
 
 
