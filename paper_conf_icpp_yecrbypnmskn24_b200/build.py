@@ -36,13 +36,16 @@ def _stale(target, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build_viper(force: bool = False, verbose: bool = False) -> str:
+def build_viper(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """defines: extra -D flags (tuning experiments build side variants via `out`)."""
+    target = out or LIB
     deps = [os.path.join(CSRC, s) for s in SOURCES + HEADERS] + [os.path.join(ROOT, "include", "viper.h")]
-    if not force and not _stale(LIB, deps):
-        return LIB
-    bdir = os.path.join(PKG, "build")
+    if not force and not _stale(target, deps):
+        return target
+    bdir = os.path.join(PKG, "build" if out is None else "build-" + os.path.basename(out))
     os.makedirs(bdir, exist_ok=True)
     common = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall", "-I", os.path.join(ROOT, "include")]
+    common += [f"-D{d}" for d in defines]
     procs, objs = [], []
     for s in SOURCES:
         o = os.path.join(bdir, s + ".o")
@@ -52,18 +55,18 @@ def build_viper(force: bool = False, verbose: bool = False) -> str:
             cmd += ["-Xptxas", "-v"] if verbose else []
         procs.append((cmd, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
     for cmd, p in procs:
-        out = p.communicate()[0].decode()
+        log = p.communicate()[0].decode()
         if p.returncode != 0:
-            raise RuntimeError("build failed:\n" + " ".join(cmd) + "\n" + out)
-        if verbose and out.strip():
-            print(out)
-    tmp = LIB + f".tmp{os.getpid()}"
+            raise RuntimeError("build failed:\n" + " ".join(cmd) + "\n" + log)
+        if verbose and log.strip():
+            print(log)
+    tmp = target + f".tmp{os.getpid()}"
     cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread", "-lrt"]
     r = subprocess.run(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)
     if r.returncode != 0:
         raise RuntimeError("link failed:\n" + r.stdout.decode())
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 def build_vgen(force: bool = False) -> str:

@@ -25,9 +25,18 @@ namespace vp {
 
 namespace {
 
-constexpr int kWarpsPerBlock = 16;   // 512 threads
-constexpr int kBlocksPerSM = 2;      // 1024 threads / SM resident
-constexpr int kUnroll = 4;           // 16-B vectors in flight per lane per step
+#ifndef VP_WARPS_PER_BLOCK
+#define VP_WARPS_PER_BLOCK 8
+#endif
+#ifndef VP_BLOCKS_PER_SM
+#define VP_BLOCKS_PER_SM 2
+#endif
+#ifndef VP_UNROLL
+#define VP_UNROLL 8
+#endif
+constexpr int kWarpsPerBlock = VP_WARPS_PER_BLOCK;  // 256 threads
+constexpr int kBlocksPerSM = VP_BLOCKS_PER_SM;      // 512 threads / SM resident (128-reg budget)
+constexpr int kUnroll = VP_UNROLL;                  // 16-B vectors in flight per lane per step
 
 __device__ __forceinline__ uint4 ld_stream(const void *p) {
     uint4 r;

@@ -10,7 +10,7 @@ import os
 import threading
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libviper.so")
+LIB_PATH = os.environ.get("VIPER_LIB_PATH") or os.path.join(_HERE, "libviper.so")  # override: tuning variants
 
 OK, E_INVAL, E_NOMEM, E_CUDA, E_VERSION, E_CHECKSUM, E_TIMEOUT, E_NOVERSION, E_STATE, E_UNSUPPORTED, E_PEER = (
     0, -1, -2, -3, -4, -5, -6, -7, -8, -9, -10)

@@ -1,6 +1,6 @@
-"""Kernel-only times of pack_seal / install_verify: the stream is kept busy
-with a sleep kernel while publish() enqueues, so the library's CUDA events
-bracket back-to-back device work (no host launch gaps inside)."""
+"""Kernel-only times: fused SYNC kernel and separate pack / install kernels.
+The stream is kept busy with a sleep kernel while publish() enqueues, so the
+library's CUDA events bracket back-to-back device work (no host launch gaps)."""
 import argparse
 import os
 import statistics
@@ -15,34 +15,39 @@ from synth import gpu as G
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="ptychonn")
-ap.add_argument("--steps", type=int, default=20)
+ap.add_argument("--steps", type=int, default=10)
 ap.add_argument("--flush", type=int, default=1)
 a = ap.parse_args()
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
-c = V.Model("kt", V.CONSUMER, ct, flags=V.FLAG_TIMING)
-p = V.Model("kt", V.PRODUCER, pt, flags=V.FLAG_TIMING)
-st = torch.cuda.current_stream()
-pk, ins, tot = [], [], []
-e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-for v in range(1, a.steps + 6):
-    G.fill_model(pt, specs, seed, v, stream=st)
-    if a.flush:
-        G.l2_flush(flush, stream=st)
-    torch.cuda._sleep(200_000)   # ~100 us: publish() enqueues behind it
-    e0.record(st)
-    p.publish(v, stream=st)
-    e1.record(st)
-    e1.synchronize()
-    if v > 5:
-        pk.append(p.stats()["t_pack_dev_us"])
-        ins.append(c.stats()["t_install_dev_us"])
-        tot.append(e0.elapsed_time(e1) * 1e3)
 S = synth.model_bytes(a.config)
-print(f"{a.config}: pack {statistics.median(pk):.2f} us ({2*S/statistics.median(pk)/1e3:.0f} GB/s)  "
-      f"install {statistics.median(ins):.2f} us ({2*S/statistics.median(ins)/1e3:.0f} GB/s)  "
-      f"pack+install back-to-back {statistics.median(tot):.2f} us  flush={a.flush}")
-c.close()
-p.close()
+res = {}
+for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE)):
+    c = V.Model("kt" + label, V.CONSUMER, ct, flags=V.FLAG_TIMING)
+    p = V.Model("kt" + label, V.PRODUCER, pt, flags=V.FLAG_TIMING | flags)
+    st = torch.cuda.current_stream()
+    fu, pk, ins = [], [], []
+    for v in range(1, a.steps + 4):
+        G.fill_model(pt, specs, seed, v, stream=st)
+        if a.flush:
+            G.l2_flush(flush, stream=st)
+        torch.cuda._sleep(400_000)
+        p.publish(v, stream=st)
+        torch.cuda.synchronize()
+        if v > 3:
+            s = p.stats()
+            fu.append(s["t_fused_dev_us"])
+            pk.append(s["t_pack_dev_us"])
+            ins.append(c.stats()["t_install_dev_us"])
+    c.close()
+    p.close()
+    if label == "fused":
+        res["fused"] = statistics.median(fu)
+    else:
+        res["pack"], res["install"] = statistics.median(pk), statistics.median(ins)
+lib = os.path.basename(os.environ.get("VIPER_LIB_PATH", "libviper.so"))
+print(f"{lib:28s} {a.config:9s} fused {res['fused']:9.2f} us ({3*S/res['fused']/1e3/6550.4:.3f})  "
+      f"pack {res['pack']:9.2f} us ({2*S/res['pack']/1e3/6550.4:.3f})  "
+      f"install {res['install']:9.2f} us ({2*S/res['install']/1e3/6550.4:.3f})", flush=True)
