@@ -70,6 +70,14 @@ def test_xproc_early_notify_pipeline(nproc, fanout, mode):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("nproc,fanout", [(3, 0), (4, 2)])
+def test_xproc_no_torn_reads(nproc, fanout):
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py", ["--config", "small", "--mode", "1", "--fanout",
+                                                           str(fanout), "--stress", "1", "--versions", "200"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 def test_xproc_fault_injection():
     rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fault", "1", "--versions", "3"])
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]

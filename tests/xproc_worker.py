@@ -27,6 +27,48 @@ def host_bytes(t):
     return t.contiguous().view(torch.uint8).reshape(-1).cpu().numpy() if t.numel() else np.zeros(0, np.uint8)
 
 
+def stress(m, rank, specs, seed, tensors, n, dev):
+    """Producer: n ASYNC publishes back to back.  Consumers: acquire -> compare
+    every byte of the view with VGEN(view.version) on the GPU -> release, until
+    the last version is seen (torn / mixed-version reads and regressions count
+    as errors)."""
+    errors = 0
+    dist.barrier()
+    if rank == 0:
+        st = torch.cuda.Stream()
+        for v in range(1, n + 1):
+            with torch.cuda.stream(st):
+                G.fill_model(tensors, specs, seed, v, stream=st)
+                m.publish(v, stream=st)
+        st.synchronize()
+    else:
+        exp = G.alloc_model(specs, device=f"cuda:{dev}")
+        s = torch.cuda.Stream()
+        last, seen = 0, 0
+        while last < n:
+            try:
+                view = m.acquire_latest(timeout_us=2_000_000)
+            except V.ViperError:
+                continue
+            with torch.cuda.stream(s):
+                G.fill_model(exp, specs, seed, view.version, stream=s)
+                got = view.tensors(tensors)
+                bad = sum(int((g.view(torch.uint8) != e.view(torch.uint8)).sum()) for g, e in zip(got, exp))
+            m.release(view, stream=s)
+            s.synchronize()
+            if bad:
+                print(f"[rank{rank}] torn view v{view.version}: {bad} bytes", flush=True)
+                errors += 1
+            if view.version < last:
+                errors += 1
+            last = view.version
+            seen += 1
+        print(f"[rank{rank}] stress: {seen} verified views, last v{last}, stats {m.stats()['installs']} installs "
+              f"{m.stats()['skipped']} skipped", flush=True)
+    dist.barrier()
+    return errors
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="ptychonn")
@@ -35,6 +77,7 @@ def main():
     ap.add_argument("--fanout", type=int, default=0)
     ap.add_argument("--versions", type=int, default=6)
     ap.add_argument("--fault", type=int, default=0)
+    ap.add_argument("--stress", type=int, default=0, help="ASYNC publishes while consumers verify every view")
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
@@ -50,6 +93,9 @@ def main():
                 bootstrap=bs)
     errors = 0
     last = 0
+    if a.stress:
+        errors += stress(m, rank, specs, seed, tensors, a.versions, dev)
+        a.versions = 0  # skip the lock-step loop
     for v in range(1, a.versions + 1):
         if a.fault and rank == 1 and v == 2:
             m.fault_next()
@@ -90,7 +136,7 @@ def main():
                     break
             m.release(view)
         dist.barrier()
-    if rank != 0 and a.mode == V.ASYNC:
+    if rank != 0 and a.mode == V.ASYNC and not a.stress:
         m.wait_installed(a.versions, timeout_us=20_000_000)
         view = m.acquire_latest()
         if view.version != a.versions:
