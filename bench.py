@@ -255,6 +255,86 @@ def c5_schedule(V, G, synth, flush, gpu_row):
     return res
 
 
+def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
+    """BASELINE.json configs[2] in 1-GPU loopback: ViT-B/16 bf16 consumer serving
+    while ASYNC updates land.  A reader thread loops acquire -> read every weight
+    byte and compare with VGEN(view.version) on the GPU (a bandwidth-heavy
+    stand-in for inference) -> stream-ordered release.  Reports
+    verified views/s without and with publishes every `period_ms`, torn views
+    (must be 0) and the install latency seen by the consumer."""
+    import threading
+    import torch
+    name = "vit_b16"
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    pt, ct = G.alloc_model(specs), G.alloc_model(specs)
+    mname = f"c3-{os.getpid()}-{time.monotonic_ns()}"
+    cons = V.Model(mname, V.CONSUMER, ct)
+    prod = V.Model(mname, V.PRODUCER, pt, mode=V.ASYNC)
+    G.fill_model(pt, specs, seed, 1)
+    prod.publish(1)
+    cons.wait_installed(1)
+    stop = threading.Event()
+    stats = {"views": 0, "torn": 0, "regress": 0}
+
+    def reader():
+        torch.cuda.set_device(torch.cuda.current_device())
+        s = torch.cuda.Stream()
+        exp = G.alloc_model(specs)
+        last = 0
+        with torch.cuda.stream(s):
+            while not stop.is_set():
+                view = cons.acquire_latest(timeout_us=100_000)
+                G.fill_model(exp, specs, seed, view.version, stream=s)
+                bad = torch.zeros((), dtype=torch.int64, device="cuda")
+                for g, e in zip(view.tensors(ct), exp):
+                    bad += (g.view(torch.uint8) != e.view(torch.uint8)).sum()
+                cons.release(view, stream=s)
+                torn = int(bad.item())
+                stats["torn"] += int(torn > 0)
+                stats["regress"] += int(view.version < last)
+                last = view.version
+                stats["views"] += 1
+
+    def phase(publish):
+        stats["views"] = 0
+        th = threading.Thread(target=reader)
+        th.start()
+        t0 = time.perf_counter()
+        v = prod.stats()["version"]
+        ps = torch.cuda.Stream()
+        n = 0
+        while time.perf_counter() - t0 < seconds:
+            if publish:
+                v += 1
+                with torch.cuda.stream(ps):
+                    G.fill_model(pt, specs, seed, v, stream=ps)
+                    prod.publish(v, stream=ps)
+                n += 1
+            time.sleep(period_ms / 1e3)
+        stop.set()
+        th.join()
+        stop.clear()
+        return stats["views"] / (time.perf_counter() - t0), n
+
+    try:
+        base, _ = phase(False)
+        busy, npub = phase(True)
+        cons.wait_installed(prod.stats()["version"])
+        cst = cons.stats()
+    finally:
+        cons.close()
+        prod.close()
+    return {"workload": "vit_b16 bf16 1 producer -> 1 consumer (1-GPU loopback), ASYNC, publish every "
+                        f"{period_ms} ms", "reader": "acquire -> byte-compare every weight with VGEN -> release",
+            "views_per_s_idle": round(base, 1), "views_per_s_during_updates": round(busy, 1),
+            "throughput_drop": round(1 - busy / base, 4) if base else None, "publishes": npub,
+            "installs": cst["installs"], "skipped": cst["skipped"], "torn_views": stats["torn"],
+            "version_regressions": stats["regress"], "last_install_us": round(cst["t_install_us"], 1),
+            "last_pickup_us": round(cst["t_notify_us"], 1),
+            "pickup_note": "publish -> update-thread pickup, includes waiting for the previous install"}
+
+
 def event_floor_us(G, reps=20):
     """An empty kernel bracketed exactly like the library's timing events."""
     import torch
@@ -513,6 +593,10 @@ def gpu_arm(args):
                     sweep[nm] = {"error": str(ex)[:200]}
                 torch.cuda.empty_cache()
             out["loopback_sweep"] = sweep
+            try:
+                out["c3_concurrent"] = c3_concurrent(V, G, synth)
+            except Exception as ex:
+                out["c3_concurrent"] = {"error": str(ex)[:200]}
             try:
                 out["c5_schedule"] = c5_schedule(V, G, synth, flush, sweep.get("llama3_8b", {}))
             except Exception as ex:
