@@ -98,8 +98,16 @@ enum { VIPER_SYNC = 0,   /* publish returns after every consumer installed v (or
 enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install
                                     kernels on their launch streams; the device
                                     times appear in viper_stats (bench.py)       */
-       VIPER_FLAG_NO_FUSE = 4 }; /* producer: never use the fused SYNC kernel
+       VIPER_FLAG_NO_FUSE = 4,   /* producer: never use the fused SYNC kernel
                                     (pack and install as separate kernels)      */
+       VIPER_FLAG_TMA = 8,       /* producer: pack through TMA bulk copies
+                                    (cp.async.bulk global<->shared) instead of
+                                    128-bit register streaming; implies NO_FUSE.
+                                    Without the flag the TMA pack is picked
+                                    automatically for packs not PDL-chained to an
+                                    install (ASYNC, DRAM tier, cross-process) of
+                                    models <= 1 GiB, where it measured faster  */
+       VIPER_FLAG_NO_TMA = 16 }; /* producer: never auto-select the TMA pack     */
 
 typedef struct {
     int32_t tier;            /* VIPER_TIER_*                       (default GPU)    */

@@ -425,6 +425,157 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fus
     }
 }
 
+// ---------------------------------------------------------------------------
+// pack_seal, TMA bulk-copy variant (VIPER_FLAG_TMA): per warp, a ring of
+// kTmaStages shared-memory stages of kTmaStage bytes.  Lane 0 streams each
+// item's 16-B-aligned body through the ring with cp.async.bulk (global ->
+// shared, mbarrier complete_tx) and cp.async.bulk (shared -> global,
+// bulk_group); all lanes checksum the stage from shared memory in between.
+// Unaligned items / <16-B tails use the register path.  Used without PDL:
+// the consumer's kernel starts after this grid completed, which makes every
+// bulk store visible.
+constexpr int kTmaStages = 3;
+constexpr uint32_t kTmaStage = 4096;
+constexpr int kTmaWarps = 8;
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(void *smem, const void *gmem, uint32_t bytes, uint64_t *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(smem)), "l"(gmem), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_s2g(void *gmem, const void *smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gmem), "r"(smem_u32(smem)),
+                 "r"(bytes)
+                 : "memory");
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+struct TmaCursor {  // position in this warp's (item, stage-sized piece) sequence
+    uint32_t w;     // item index
+    uint32_t off;   // byte offset inside the item's TMA body
+};
+
+__device__ __forceinline__ uint32_t tma_body(const Item &it) {
+    // TMA needs 16-B aligned addresses and sizes; the rest goes through registers
+    return ((it.ptr | it.packed_off) & 15u) ? 0u : (it.nbytes & ~15u);
+}
+
+__global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const PackArgs a) {
+    extern __shared__ __align__(128) uint8_t tma_smem[];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    uint8_t *stage = tma_smem + wib * (kTmaStages * kTmaStage);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(tma_smem + kTmaWarps * kTmaStages * kTmaStage) + wib * kTmaStages;
+    if (lane == 0) {
+        for (int s = 0; s < kTmaStages; s++) mbar_init(bar + s);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    const uint32_t nwarps = gridDim.x * kTmaWarps;
+    const uint32_t w0 = blockIdx.x * kTmaWarps + wib;
+    // loader cursor: the next piece to bring in; skips items without a TMA body
+    TmaCursor ld{w0, 0};
+    auto next_piece = [&](TmaCursor &c, Item &it, uint32_t &bytes) -> bool {
+        while (c.w < a.nitems) {
+            it = a.items[c.w];
+            const uint32_t body = tma_body(it);
+            if (c.off < body) {
+                bytes = min(kTmaStage, body - c.off);
+                return true;
+            }
+            c.w += nwarps;
+            c.off = 0;
+        }
+        return false;
+    };
+    uint32_t issued = 0, phase_bits = 0;
+    // prologue: fill the ring
+    for (int s = 0; s < kTmaStages; s++) {
+        Item it;
+        uint32_t bytes;
+        if (!next_piece(ld, it, bytes)) break;
+        if (lane == 0) {
+            mbar_expect_tx(bar + s, bytes);
+            bulk_g2s(stage + s * kTmaStage, (const uint8_t *)it.ptr + ld.off, bytes, bar + s);
+        }
+        ld.off += bytes;
+        issued++;
+    }
+    uint32_t consumed = 0;
+    for (uint32_t w = w0; w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        const uint32_t body = tma_body(it);
+        uint64_t acc = 0;
+        for (uint32_t off = 0; off < body; off += kTmaStage) {
+            const uint32_t bytes = min(kTmaStage, body - off);
+            const int s = consumed % kTmaStages;
+            mbar_wait(bar + s, (phase_bits >> s) & 1u);
+            phase_bits ^= 1u << s;
+            const uint8_t *buf = stage + s * kTmaStage;
+            const uint32_t g0 = (uint32_t)((it.packed_off + off) >> 2);
+            for (uint32_t i = lane; i < bytes / 16; i += 32)
+                acc += cks_vec(*reinterpret_cast<const uint4 *>(buf + i * 16), g0 + 4u * i);
+            __syncwarp();
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                bulk_s2g(a.packed + it.packed_off + off, buf, bytes);
+            }
+            consumed++;
+            // refill this stage with the piece kTmaStages ahead once its store has read it
+            Item nit;
+            uint32_t nbytes;
+            if (next_piece(ld, nit, nbytes)) {
+                if (lane == 0) {
+                    bulk_wait_read<0>();
+                    mbar_expect_tx(bar + s, nbytes);
+                    bulk_g2s(stage + s * kTmaStage, (const uint8_t *)nit.ptr + ld.off, nbytes, bar + s);
+                }
+                ld.off += nbytes;
+                issued++;
+            }
+        }
+        if (body < it.nbytes)  // unaligned item or <16-B tail: register path
+            acc += (body == 0) ? copy_item<false>((const uint8_t *)it.ptr, a.packed + it.packed_off, it.nbytes,
+                                                  it.packed_off, lane, false)
+                               : copy_words_bytewise<false>((const uint8_t *)it.ptr + 0, a.packed + it.packed_off,
+                                                            body, it.nbytes, it.packed_off, lane, false);
+        const uint64_t part = warp_sum(acc);
+        if (lane == 0) {
+            a.iseal[w].mixed = part + a.version * kVerMix;
+            a.iseal[w].version = a.version;  // visible to the next kernel (no PDL with this variant)
+        }
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    (void)issued;
+}
+
 }  // namespace
 
 Geometry pick_geometry(uint32_t nitems, int device) {
@@ -443,6 +594,22 @@ Geometry pick_geometry(uint32_t nitems, int device) {
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
     if (a.nitems == 0) return cudaSuccess;
     pack_seal_kernel<<<g.grid, g.block, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
+    if (a.nitems == 0) return cudaSuccess;
+    static int sms = 0;
+    const size_t smem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
+    if (sms == 0) {
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) sms = 148;
+        cudaError_t e = cudaFuncSetAttribute(pack_seal_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    const uint32_t want = (a.nitems + kTmaWarps - 1) / kTmaWarps;
+    const uint32_t cap = (uint32_t)sms * 2;
+    const int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+    pack_seal_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 

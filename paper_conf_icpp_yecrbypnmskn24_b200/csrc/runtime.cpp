@@ -542,8 +542,13 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     TRACE(2);
     const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
     std::vector<viper_model *> launched;
+    // TMA bulk-copy pack: forced by the flag, or auto for packs no install is
+    // PDL-chained to (profiles/r01: faster up to ~1 GB, slightly slower above)
+    const bool tma_auto = !(p->cfg.flags & VIPER_FLAG_NO_TMA) && (!sync || dram || p->xproc) &&
+                          p->man.s_packed <= (1ull << 30);
+    const bool tma = ((p->cfg.flags & VIPER_FLAG_TMA) || tma_auto) && !p->early_notify;
     const bool fuse = sync && !dram && !prepared.empty() && prepared.size() <= (size_t)kMaxFused &&
-                      !(p->cfg.flags & VIPER_FLAG_NO_FUSE);
+                      !(p->cfg.flags & (VIPER_FLAG_NO_FUSE | VIPER_FLAG_TMA));
     if (fuse) {
         // one kernel: pack + seal + install + verify + swap for every local consumer
         FusedArgs f{};
@@ -579,7 +584,8 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         a.version = v;
         a.sys_release = p->early_notify ? 1u : 0u;
         if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
-        CUDA_TRY(launch_pack(a, p->geo, st));
+        if (tma) CUDA_TRY(launch_pack_tma(a, st, p->device));
+        else CUDA_TRY(launch_pack(a, p->geo, st));
         if (timing) {
             CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
             p->timing_pending = true;
@@ -588,7 +594,9 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     p->last_fused = fuse;
     auto launch_all = [&]() {
         for (PreparedInstall &pi : prepared) {
-            viper_status s = launch_prepared(pi, psrc, b, st, dram, !dram && launched.empty());
+            // PDL item pipeline behind the register-path pack only (the TMA
+            // pack's stores are visible at grid completion)
+            viper_status s = launch_prepared(pi, psrc, b, st, dram, !dram && !tma && launched.empty());
             if (s != VIPER_OK) {
                 result = s;
                 continue;

@@ -121,6 +121,8 @@ struct Geometry {
 Geometry pick_geometry(uint32_t nitems, int device);
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
+// TMA bulk-copy pack (cp.async.bulk); consumers must not be PDL-chained to it
+cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device);
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
 // pdl: the install directly follows the pack on `st` (programmatic dependent launch)

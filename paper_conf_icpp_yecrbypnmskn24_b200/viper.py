@@ -21,6 +21,8 @@ FANOUT_DIRECT, FANOUT_SCATTER_ALLGATHER = 0, 2
 SYNC, ASYNC = 0, 1
 FLAG_TIMING = 2
 FLAG_NO_FUSE = 4
+FLAG_TMA = 8
+FLAG_NO_TMA = 16
 SCHED_FIXED, SCHED_GREEDY = 0, 1
 
 

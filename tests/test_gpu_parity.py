@@ -78,6 +78,7 @@ def close_all(prod, cons):
 
 # ------------------------------------------------------------------ C1 (BJ configs[0])
 @pytest.mark.parametrize("tier,mode,flags", [(V.TIER_GPU, V.SYNC, 0), (V.TIER_GPU, V.SYNC, V.FLAG_NO_FUSE),
+                                              (V.TIER_GPU, V.SYNC, V.FLAG_TMA), (V.TIER_GPU, V.ASYNC, V.FLAG_TMA),
                                               (V.TIER_GPU, V.ASYNC, 0), (V.TIER_DRAM, V.SYNC, 0),
                                               (V.TIER_DRAM, V.ASYNC, 0)])
 def test_c1_ptychonn_10_versions(tier, mode, flags):
@@ -118,7 +119,7 @@ def test_ragged_tensor_lists_many_chunks(seed):
         specs.append((f"t{i}", dt, (ne,)))
     chunk = int(rng.choice([256, 4096, 65536]))
     align = int(rng.choice([16, 256]))
-    flags = V.FLAG_NO_FUSE if seed % 2 else 0
+    flags = [0, V.FLAG_NO_FUSE, V.FLAG_TMA][seed % 3]
     ncons = 3 if seed < 4 else 6   # > kMaxFused local consumers -> separate kernels
     prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=ncons, chunk_bytes=chunk, align=align, flags=flags)
     try:
@@ -348,15 +349,16 @@ def test_no_torn_reads_under_async_publishes():
 
 
 # ----------------------------------------------- BJ-sized models in 1-GPU loopback
-@pytest.mark.parametrize("name", ["resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
-def test_full_size_loopback_sampled(name):
+@pytest.mark.parametrize("name,flags", [("resnet50", 0), ("vit_b16", 0), ("gpt2_xl", 0), ("llama3_8b", 0),
+                                        ("gpt2_xl", V.FLAG_TMA)])
+def test_full_size_loopback_sampled(name, flags):
     """Full BASELINE.json model sizes, single-GPU loopback (the launch config
     bench.py times): every seal's version; sampled chunk seals recomputed by the
     oracle; sampled tensor byte ranges vs VGEN; all slot tensors == producer
     tensors (replica identity at any size)."""
     specs = synth.model_specs(name)
     seed = synth.SEEDS[name]
-    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.SYNC)
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.SYNC, flags=flags)
     try:
         for v in (1, 2):
             G.fill_model(prod_t, specs, seed, v)

@@ -24,7 +24,7 @@ pt, ct = G.alloc_model(specs), G.alloc_model(specs)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 S = synth.model_bytes(a.config)
 res = {}
-for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE)):
+for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE), ("tma", V.FLAG_TMA)):
     c = V.Model("kt" + label, V.CONSUMER, ct, flags=V.FLAG_TIMING)
     p = V.Model("kt" + label, V.PRODUCER, pt, flags=V.FLAG_TIMING | flags)
     st = torch.cuda.current_stream()
@@ -45,9 +45,12 @@ for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE)):
     p.close()
     if label == "fused":
         res["fused"] = statistics.median(fu)
-    else:
+    elif label == "sep":
         res["pack"], res["install"] = statistics.median(pk), statistics.median(ins)
+    else:
+        res["tma"] = statistics.median(pk)
 lib = os.path.basename(os.environ.get("VIPER_LIB_PATH", "libviper.so"))
 print(f"{lib:28s} {a.config:9s} fused {res['fused']:9.2f} us ({3*S/res['fused']/1e3/6550.4:.3f})  "
       f"pack {res['pack']:9.2f} us ({2*S/res['pack']/1e3/6550.4:.3f})  "
-      f"install {res['install']:9.2f} us ({2*S/res['install']/1e3/6550.4:.3f})", flush=True)
+      f"install {res['install']:9.2f} us ({2*S/res['install']/1e3/6550.4:.3f})  "
+      f"pack_tma {res['tma']:9.2f} us ({2*S/res['tma']/1e3/6550.4:.3f})", flush=True)
