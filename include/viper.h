@@ -80,6 +80,13 @@ typedef struct {
     int32_t rank, world, producer_rank;
     int (*allgather)(const void *in, void *out, size_t nbytes, void *user);
     void *user;
+    /* Data-parallel producers ("multiple producers running
+     * data-parallel training"): ranks producer_rank ..
+     * producer_rank + nproducers - 1 are producers holding identical replicas;
+     * each publishes the same versions and packs only the chunks c with
+     * c % nproducers == its index, consumers pull every chunk from its owner.
+     * 0 or 1 = a single producer.  GPU tier, direct fan-out only. */
+    int32_t nproducers;
 } viper_bootstrap;
 
 /* Storage tier (s4.4 P:1671-1720, Fig. 7). */

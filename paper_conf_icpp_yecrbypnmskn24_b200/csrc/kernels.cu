@@ -237,9 +237,10 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
                                                         it.nbytes, it.packed_off, lane, false));
         __syncwarp();  // every lane's stores are ordered before lane 0's release
         if (lane == 0) {
-            a.iseal[w].mixed = part + a.version * kVerMix;
-            if (a.sys_release) st_release_sys(&a.iseal[w].version, a.version);  // readers on other GPUs
-            else st_release(&a.iseal[w].version, a.version);  // item w ready (pipelined install)
+            ISeal *is = a.iseal + it.gidx;
+            is->mixed = part + a.version * kVerMix;
+            if (a.sys_release) st_release_sys(&is->version, a.version);  // readers on other GPUs
+            else st_release(&is->version, a.version);  // item ready (pipelined install)
         }
     }
 }
@@ -250,6 +251,7 @@ __global__ void seal_reduce_kernel(const SealReduceArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t c = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     if (c >= a.nchunks) return;
+    if (a.share_n > 1 && c % a.share_n != a.share_me) return;  // another producer's chunk
     const uint32_t lo = a.chunk_first[c], hi = a.chunk_first[c + 1];
     uint64_t s = 0;
     for (uint32_t i = lo + lane; i < hi; i += 32) s += a.iseal[i].mixed - a.version * kVerMix;
@@ -278,6 +280,11 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
         // with L2-coherent loads.  Without PDL the flag is already set.
         const uint8_t *src = a.packed + it.packed_off;
         const ISeal *is = a.iseal + w;
+        if (a.mp_n > 1) {  // data-parallel producers: the chunk's owner packed it
+            const uint32_t p = it.chunk % a.mp_n;
+            src = a.mp_snap[p] + it.packed_off;
+            is = a.mp_iseal[p] + w;
+        }
         uint32_t owner = a.sa_n ? it.chunk % a.sa_n : 0;
         if (a.sa_n && owner != a.sa_me) {
             // scatter-allgather: the owner re-publishes this item in its staging
@@ -568,8 +575,8 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const 
                                                             body, it.nbytes, it.packed_off, lane, false);
         const uint64_t part = warp_sum(acc);
         if (lane == 0) {
-            a.iseal[w].mixed = part + a.version * kVerMix;
-            a.iseal[w].version = a.version;  // visible to the next kernel (no PDL with this variant)
+            a.iseal[it.gidx].mixed = part + a.version * kVerMix;
+            a.iseal[it.gidx].version = a.version;  // visible to the next kernel (no PDL with this variant)
         }
     }
     if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");

@@ -166,14 +166,19 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
 
 // Device work list of one endpoint: the base items with that endpoint's tensor
 // addresses folded in.
-viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out) {
+viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out, uint32_t share_n,
+                          uint32_t share_me, uint32_t *count) {
     *d_out = nullptr;
-    if (m.items.empty()) return VIPER_OK;
-    std::vector<Item> v(m.items.size());
-    for (size_t k = 0; k < v.size(); k++) {
+    std::vector<Item> v;
+    v.reserve(m.items.size());
+    for (size_t k = 0; k < m.items.size(); k++) {
         const BaseItem &b = m.items[k];
-        v[k] = Item{(uint64_t)(uintptr_t)ptrs[b.tensor] + b.tensor_off, b.packed_off, b.nbytes, b.chunk, b.tensor, 0};
+        if (share_n > 1 && b.chunk % share_n != share_me) continue;  // another producer's chunk
+        v.push_back(Item{(uint64_t)(uintptr_t)ptrs[b.tensor] + b.tensor_off, b.packed_off, b.nbytes, b.chunk, b.tensor,
+                         (uint32_t)k});
     }
+    if (count) *count = (uint32_t)v.size();
+    if (v.empty()) return VIPER_OK;
     CUDA_TRY(cudaMalloc((void **)d_out, v.size() * sizeof(Item)));
     CUDA_TRY(cudaMemcpy(*d_out, v.data(), v.size() * sizeof(Item), cudaMemcpyHostToDevice));
     return VIPER_OK;
@@ -233,6 +238,34 @@ void fire_callback(viper_model *c, uint64_t v, viper_status st) {
 // Pin the latest published snapshot (Dekker pair with the producer's
 // pub_state store -> pin scan).  Returns false when
 // nothing is published.
+// Multi-producer: the version every producer published (all pub_m equal).
+static bool all_published(Ctrl *ctrl, int M, uint64_t *word) {
+    const uint64_t w0 = ctrl->pub_m[0].load();
+    for (int j = 1; j < M; j++)
+        if (ctrl->pub_m[j].load() != w0) return false;
+    *word = w0;
+    return w0 != 0;
+}
+
+bool pin_latest_m(Ctrl *ctrl, ConsRec *r, int M, uint64_t *v, int *b) {
+    for (int tries = 0; tries < 1000; tries++) {
+        uint64_t w;
+        if (!all_published(ctrl, M, &w)) {
+            sched_yield();
+            continue;
+        }
+        r->pin.store(w >> 1);
+        uint64_t w2;
+        if (all_published(ctrl, M, &w2) && w2 == w) {
+            *v = w >> 1;
+            *b = (int)(w & 1);
+            return true;
+        }
+        r->pin.store(0);
+    }
+    return false;
+}
+
 bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
     for (;;) {
         const uint64_t ps = ctrl->pub_state.load();
@@ -373,7 +406,8 @@ void update_loop(viper_model *c) {
     ConsRec *r = c->rec;
     while (!c->stop.load()) {
         const uint32_t seq = ctrl->pub_seq.load();
-        const uint64_t ps = ctrl->pub_state.load();
+        uint64_t ps = ctrl->pub_state.load();
+        if (c->nprod > 1 && !all_published(ctrl, c->nprod, &ps)) ps = 0;
         bool work;
         {
             // SYNC producers install inline; the thread only catches a consumer
@@ -404,7 +438,7 @@ void update_loop(viper_model *c) {
         std::unique_lock<std::mutex> lk(c->install_mu);
         uint64_t v;
         int b;
-        if (!pin_latest(ctrl, r, &v, &b)) continue;
+        if (!(c->nprod > 1 ? pin_latest_m(ctrl, r, c->nprod, &v, &b) : pin_latest(ctrl, r, &v, &b))) continue;
         if (v <= c->attempted) {
             r->pin.store(0);
             continue;
@@ -470,6 +504,10 @@ viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
 int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug_trace)
 #define TRACE(i) (g_trace[i] = now_ns())
 
+std::atomic<uint64_t> &pub_word(viper_model *p) {
+    return p->nprod > 1 ? p->ctrl->pub_m[p->pidx] : p->ctrl->pub_state;
+}
+
 static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st) {
     const int64_t t0 = now_ns();
     g_trace[0] = t0;
@@ -481,7 +519,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // ASYNC cross-process: the previous version's notification (a host
         // function after its pack) must have named it before slot reuse
         const int64_t w0 = now_ns();
-        while ((ctrl->pub_state.load() >> 1) != p->last_version) {
+        while ((pub_word(p).load() >> 1) != p->last_version) {
             if (now_ns() - w0 > 60ll * 1000000000ll) return set_error(VIPER_E_TIMEOUT, "previous publish stuck");
             sched_yield();
         }
@@ -578,7 +616,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     } else {
         PackArgs a{};
         a.items = p->d_items;
-        a.nitems = (uint32_t)p->man.items.size();
+        a.nitems = p->pack_nitems;  // this producer's chunk share (all items with one producer)
         a.packed = p->d_snap[b];
         a.iseal = p->d_iseal[b];
         a.version = v;
@@ -614,7 +652,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // in process, consumers order themselves after ev_ready[b]; across
         // GPUs with early notification their install waits per item on the
         // seals the pack releases at system scope (cross-GPU pipeline)
-        ctrl->pub_state.store((v << 1) | (uint64_t)b);
+        pub_word(p).store((v << 1) | (uint64_t)b);
         ctrl->pub_time_ns.store(now_ns());
         if (p->xproc) {
             ctrl->pub_seq.fetch_add(1);
@@ -654,6 +692,8 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     ra.iseal = p->d_iseal[b];
     ra.seals = p->d_seal[b];
     ra.version = v;
+    ra.share_n = (uint32_t)p->nprod;
+    ra.share_me = (uint32_t)p->pidx;
     CUDA_TRY(launch_seal_reduce(ra, p->side));
     CUDA_TRY(cudaEventRecord(p->ev_sealed[b], p->side));
     TRACE(4);
@@ -754,7 +794,8 @@ viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) {
     const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
     const uint64_t CS = al256(sizeof(Seal) * std::max<uint32_t>(m->man.nchunks, 1));
     for (int32_t i = 0; i < m->man.n; i++) m->src_ptrs.push_back(tensors[i].dev_ptr);
-    viper_status st = upload_items(m->man, m->src_ptrs, &m->d_items);
+    viper_status st = upload_items(m->man, m->src_ptrs, &m->d_items, (uint32_t)m->nprod, (uint32_t)m->pidx,
+                                   &m->pack_nitems);
     if (st) return st;
     const size_t bytes = 2 * (S + IS + CS);
     CUDA_TRY(cudaMalloc(&m->snap_alloc, bytes));
@@ -800,7 +841,7 @@ viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
         for (int32_t i = 0; i < m->man.n; i++) m->slot_ptrs[1].push_back((uint8_t *)m->slot1_alloc + m->man.offsets[i]);
     }
     for (int s = 0; s < 2; s++)
-        if ((st = upload_items(m->man, m->slot_ptrs[s], &m->d_slot_items[s]))) return st;
+        if ((st = upload_items(m->man, m->slot_ptrs[s], &m->d_slot_items[s], 1, 0, nullptr))) return st;
     CUDA_TRY(cudaMalloc(&m->d_flags, 64));
     CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
     if (m->cfg.tier == VIPER_TIER_DRAM) {

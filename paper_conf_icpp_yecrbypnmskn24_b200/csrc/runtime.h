@@ -26,7 +26,8 @@
 namespace vp {
 
 constexpr int kMaxConsumers = 16;
-constexpr int kMaxPieces = 256;  // DRAM tier: D2H / H2D pipeline granularity (whole chunks)
+constexpr int kMaxPieces = 256;     // DRAM tier: D2H / H2D pipeline granularity (whole chunks)
+constexpr int kMaxProducers = 8;   // data-parallel producers (multi-producer fan-in)
 constexpr uint64_t kCtrlMagic = 0x5649504552435431ull;  // "VIPERCT1"
 
 struct alignas(64) ConsRec {
@@ -55,6 +56,10 @@ struct alignas(64) Ctrl {
     // dram_flag[b][i] >= v (written by the producer's copy stream with
     // cuStreamWriteValue64; consumers' copy streams wait with cuStreamWaitValue64)
     alignas(64) std::atomic<uint64_t> dram_flag[2][kMaxPieces];
+    // multi-producer: producer j's (v << 1) | slot; consumers install v once
+    // every producer published it
+    alignas(64) std::atomic<uint64_t> pub_m[kMaxProducers];
+    std::atomic<int32_t> nprod;
 };
 
 // Pointer-free work item (the device lists add each endpoint's tensor address).
@@ -168,6 +173,10 @@ struct viper_model {
     uint64_t sa_S = 0, sa_IS = 0;
     int32_t rank = 0, world = 1;
     bool early_notify = false;                       // producer: consumers pipeline behind the pack
+    int32_t nprod = 1, pidx = 0;                     // data-parallel producers / this producer's index
+    uint32_t pack_nitems = 0;                        // items this producer packs (its chunk share)
+    void *peer_snap_m[vp::kMaxProducers] = {};        // consumer: every producer's snapshot (IPC)
+    void *d_mp_tab = nullptr;                        // consumer: snap[2][M], iseal[2][M]
 
     // ---------------- stats
     std::mutex stats_mu;
@@ -198,7 +207,9 @@ void futex_wake_all(std::atomic<uint32_t> *w);
 void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us);
 viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes, uint32_t align,
                             int device);
-viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out);
+viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out, uint32_t share_n,
+                          uint32_t share_me, uint32_t *count);
+std::atomic<uint64_t> &pub_word(viper_model *p);
 bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b);
 viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, int b, PreparedInstall *pi);
 viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, cudaStream_t st, bool wait_ready,

@@ -16,7 +16,7 @@ struct Item {
     uint32_t nbytes;       // bytes of this piece (multiple of 16 except a tensor tail)
     uint32_t chunk;        // seal chunk index
     uint32_t tensor;       // tensor index
-    uint32_t pad;
+    uint32_t gidx;         // index in the full work list (item seals are indexed by it)
 };
 static_assert(sizeof(Item) == 32, "Item must stay 32 B");
 
@@ -59,6 +59,7 @@ struct SealReduceArgs {
     const ISeal *iseal;
     Seal *seals;                  // [nchunks] {version, cks} (written)
     uint64_t version;
+    uint32_t share_n, share_me;   // multi-producer: only chunks c % share_n == share_me
 };
 
 struct InstallArgs {
@@ -84,6 +85,11 @@ struct InstallArgs {
     // shows `version`, falling back to the producer when the owner is not
     // installing this version.
     uint32_t sa_n, sa_me;
+    // Multi-producer fan-in (mp_n > 1): item x comes from producer
+    // chunk(x) % mp_n (data-parallel replicas each pack their share)
+    uint32_t mp_n;
+    const uint8_t *const *mp_snap;               // [mp_n] producers' snapshot slot (device-mapped)
+    const ISeal *const *mp_iseal;                // [mp_n] producers' item seals
     uint8_t *sa_stage_out;
     ISeal *sa_iseal_out;
     const uint8_t *const *sa_src;                // [sa_n] peers' staging (device-mapped)

@@ -128,12 +128,13 @@ viper_status map_control(viper_model *m) {
 
 struct NotifyCtx {
     Ctrl *ctrl;
+    std::atomic<uint64_t> *pub;  // pub_state, or pub_m[j] for data-parallel producer j
     uint64_t word;
 };
 
 void CUDART_CB notify_fn(void *p) {  // host function: no CUDA calls here
     NotifyCtx *n = (NotifyCtx *)p;
-    n->ctrl->pub_state.store(n->word);
+    n->pub->store(n->word);
     n->ctrl->pub_time_ns.store(now_ns());
     n->ctrl->pub_seq.fetch_add(1);
     futex_wake_all(&n->ctrl->pub_seq);
@@ -146,7 +147,7 @@ viper_status open_sa_peers(viper_model *m, const std::vector<PeerRec> &all, cons
     std::vector<const volatile uint64_t *> pins(N);
     int j = 0;
     for (int r = 0; r < bs->world; r++) {
-        if (r == bs->producer_rank) continue;
+        if (all[r].role == VIPER_PRODUCER) continue;
         uint8_t *base;
         if (j == m->cidx) {
             base = (uint8_t *)m->sa_alloc;
@@ -171,17 +172,47 @@ viper_status open_sa_peers(viper_model *m, const std::vector<PeerRec> &all, cons
     return VIPER_OK;
 }
 
+// Data-parallel producers: map every producer's snapshot allocation and
+// upload the per-slot tables the install kernel indexes by chunk % M.
+viper_status open_producers(viper_model *m, const std::vector<PeerRec> &all, const viper_bootstrap *bs) {
+    const int M = m->nprod;
+    std::vector<const void *> tab(4 * M);
+    for (int j = 0; j < M; j++) {
+        const PeerRec &pj = all[bs->producer_rank + j];
+        void *base;
+        if (j == 0) {
+            base = m->peer_snap_base;  // opened above for producer 0
+        } else {
+            CUDA_TRY(cudaIpcOpenMemHandle(&m->peer_snap_m[j], pj.snap_handle, cudaIpcMemLazyEnablePeerAccess));
+            base = m->peer_snap_m[j];
+        }
+        for (int b = 0; b < 2; b++) {
+            tab[b * M + j] = (const uint8_t *)base + pj.snap_off[b];
+            tab[2 * M + b * M + j] = (const uint8_t *)base + pj.iseal_off[b];
+        }
+    }
+    CUDA_TRY(cudaMalloc(&m->d_mp_tab, tab.size() * sizeof(void *)));
+    CUDA_TRY(cudaMemcpy(m->d_mp_tab, tab.data(), tab.size() * sizeof(void *), cudaMemcpyHostToDevice));
+    return VIPER_OK;
+}
+
 }  // namespace
 
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs) {
     if (!bs->allgather) return set_error(VIPER_E_INVAL, "bootstrap.allgather is NULL");
     if (bs->rank < 0 || bs->rank >= bs->world || bs->producer_rank < 0 || bs->producer_rank >= bs->world)
         return set_error(VIPER_E_INVAL, "bad bootstrap ranks");
-    if (bs->world - 1 > kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+    const int M = bs->nproducers > 1 ? bs->nproducers : 1;
+    if (M > kMaxProducers || bs->producer_rank + M > bs->world)
+        return set_error(VIPER_E_INVAL, "bad nproducers %d", bs->nproducers);
+    if (bs->world - M > kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
     m->rank = bs->rank;
     m->world = bs->world;
-    m->nconsumers_x = bs->world - 1;
+    m->nconsumers_x = bs->world - M;
+    m->nprod = M;
     const bool producer = m->role == VIPER_PRODUCER;
+    const bool is_prod_rank = bs->rank >= bs->producer_rank && bs->rank < bs->producer_rank + M;
+    m->pidx = is_prod_rank ? bs->rank - bs->producer_rank : 0;
     const bool dram = m->cfg.tier == VIPER_TIER_DRAM;
     PeerRec me{};
     me.magic = kPeerMagic;
@@ -197,20 +228,23 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
     me.manifest_hash = manifest_hash(m->man);
     cudaDeviceGetPCIBusId(me.pci, sizeof me.pci, m->device);
     viper_status st = VIPER_OK;
-    if (producer != (bs->rank == bs->producer_rank))
-        st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank", bs->rank);
+    if (producer != is_prod_rank)
+        st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank/nproducers", bs->rank);
+    if (st == VIPER_OK && M > 1 && (m->cfg.tier != VIPER_TIER_GPU || m->cfg.fanout != VIPER_FANOUT_DIRECT))
+        st = set_error(VIPER_E_UNSUPPORTED, "data-parallel producers: GPU tier, direct fan-out only");
     const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
     const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
+    const size_t ctrl_bytes = page_up(sizeof(Ctrl));
     if (st == VIPER_OK && producer) {
         st = alloc_producer(m, tensors);
-        const size_t ctrl_bytes = page_up(sizeof(Ctrl));
         const size_t bytes = ctrl_bytes + (dram ? 2 * (S + IS) : 0);
-        if (st == VIPER_OK) st = create_segment(m, bytes, me.shm_path, sizeof me.shm_path);
-        if (st == VIPER_OK) {
+        if (st == VIPER_OK && m->pidx == 0) st = create_segment(m, bytes, me.shm_path, sizeof me.shm_path);
+        if (st == VIPER_OK && m->pidx == 0) {
             memset(m->shm_base, 0, ctrl_bytes);
             Ctrl *c = new (m->shm_base) Ctrl();
             c->magic = kCtrlMagic;
-            c->ncons.store(bs->world - 1);
+            c->ncons.store(bs->world - M);
+            c->nprod.store(M);
             st = map_control(m);
         }
         if (st == VIPER_OK) {
@@ -219,7 +253,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             for (int b = 0; b < 2; b++) {
                 me.snap_off[b] = (uint64_t)(m->d_snap[b] - (uint8_t *)m->snap_alloc);
                 me.iseal_off[b] = (uint64_t)((uint8_t *)m->d_iseal[b] - (uint8_t *)m->snap_alloc);
-                if (dram) {
+                if (dram && m->pidx == 0) {
                     me.stage_off[b] = ctrl_bytes + b * S;
                     me.hiseal_off[b] = ctrl_bytes + 2 * S + b * IS;
                     m->h_stage[b] = h + b * S;
@@ -256,19 +290,23 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
                 st = set_error(VIPER_E_INVAL, "rank %d uses another tier / fan-out", r);
         }
     }
+    if (st == VIPER_OK && producer && m->pidx > 0) {  // data-parallel producer j > 0: join the segment
+        st = open_segment(m, pr.shm_path, pr.shm_bytes);
+        if (st == VIPER_OK) st = map_control(m);
+    }
     if (st == VIPER_OK && producer) {
         // every consumer on another GPU: publish v as soon as the pack is
         // launched; consumers pull items as their seals are released (.sys)
         bool other = true;
         for (int r = 0; r < bs->world; r++)
-            if (r != bs->producer_rank && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
+            if (all[r].role != VIPER_PRODUCER && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
         const char *env = getenv("VIPER_EARLY_NOTIFY");
         m->early_notify = env ? atoi(env) != 0 : other;
     }
     if (st == VIPER_OK && !producer) {
         int idx = 0;
         for (int r = 0; r < bs->rank; r++)
-            if (r != bs->producer_rank) idx++;
+            if (all[r].role != VIPER_PRODUCER) idx++;
         m->cidx = idx;
         st = open_segment(m, pr.shm_path, pr.shm_bytes);
         if (st == VIPER_OK) st = map_control(m);
@@ -294,6 +332,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             st = alloc_consumer(m, tensors);
         }
         if (st == VIPER_OK && sa) st = open_sa_peers(m, all, bs);
+        if (st == VIPER_OK && M > 1) st = open_producers(m, all, bs);
         if (st == VIPER_OK) m->rec->active.store(1);
     }
     // ---- allgather #2: statuses (all ranks fail together)
@@ -313,6 +352,17 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
 // Consumer update thread (install_mu held, v pinned): pull slot b of the
 // producer over the peer mapping (or from the shared DRAM staging).
 viper_status xproc_install(viper_model *c, uint64_t v, int b) {
+    if (c->nprod > 1) {
+        PreparedInstall pi;
+        viper_status s = prepare_install(c, c->xsrc, v, b, &pi);
+        if (s) return s;
+        const int M = c->nprod;
+        const void *const *tab = (const void *const *)c->d_mp_tab;
+        pi.a.mp_n = (uint32_t)M;
+        pi.a.mp_snap = (const uint8_t *const *)(tab + b * M);
+        pi.a.mp_iseal = (const ISeal *const *)(tab + 2 * M + b * M);
+        return launch_prepared(pi, c->xsrc, b, c->ustream, false, false);
+    }
     if (c->cfg.fanout != VIPER_FANOUT_SCATTER_ALLGATHER || c->nconsumers_x < 2 || c->cfg.tier != VIPER_TIER_GPU)
         return enqueue_install(c, c->xsrc, v, b, c->ustream, false);
     PreparedInstall pi;
@@ -337,7 +387,7 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
     Ctrl *ctrl = p->ctrl;
     const uint64_t word = (v << 1) | (uint64_t)b;
     if (!sync) {
-        NotifyCtx *n = new NotifyCtx{ctrl, word};
+        NotifyCtx *n = new NotifyCtx{ctrl, &pub_word(p), word};
         const cudaError_t e = cudaLaunchHostFunc(p->side, notify_fn, n);
         if (e != cudaSuccess) {
             delete n;
@@ -347,7 +397,7 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
     }
     if (!already) {
         CUDA_TRY(cudaEventSynchronize(p->ev_packed));
-        ctrl->pub_state.store(word);
+        pub_word(p).store(word);
         ctrl->pub_time_ns.store(now_ns());
         ctrl->pub_seq.fetch_add(1);
         futex_wake_all(&ctrl->pub_seq);
@@ -377,6 +427,10 @@ void xproc_free(viper_model *m) {
     if (m->role == VIPER_PRODUCER && m->ctrl) m->ctrl->closing.store(1);
     for (auto &p : m->sa_peer_base)
         if (p) cudaIpcCloseMemHandle(p), p = nullptr;
+    for (auto &p : m->peer_snap_m)
+        if (p) cudaIpcCloseMemHandle(p), p = nullptr;
+    cudaFree(m->d_mp_tab);
+    m->d_mp_tab = nullptr;
     cudaFree(m->d_sa_tab);
     cudaFree(m->sa_alloc);
     m->d_sa_tab = m->sa_alloc = nullptr;

@@ -36,7 +36,7 @@ ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void
 
 class viper_bootstrap(C.Structure):
     _fields_ = [("rank", C.c_int32), ("world", C.c_int32), ("producer_rank", C.c_int32),
-                ("allgather", ALLGATHER_FN), ("user", C.c_void_p)]
+                ("allgather", ALLGATHER_FN), ("user", C.c_void_p), ("nproducers", C.c_int32)]
 
 
 class viper_config(C.Structure):
@@ -274,8 +274,11 @@ def _stream_ptr(stream):
 class Bootstrap:
     """Cross-process bootstrap over a torch.distributed process group."""
 
-    def __init__(self, rank: int, world: int, producer_rank: int = 0, group=None):
+    def __init__(self, rank: int, world: int, producer_rank: int = 0, group=None, nproducers: int = 1):
+        """nproducers > 1: ranks producer_rank .. producer_rank+nproducers-1 are
+        data-parallel producers, each packing its share of the chunks."""
         self.rank, self.world, self.producer_rank, self.group = rank, world, producer_rank, group
+        self.nproducers = nproducers
 
     def _allgather(self, inp, out, nbytes, user):
         try:
@@ -296,7 +299,7 @@ class Bootstrap:
 
     def struct(self) -> viper_bootstrap:
         self._fn = ALLGATHER_FN(self._allgather)
-        return viper_bootstrap(self.rank, self.world, self.producer_rank, self._fn, None)
+        return viper_bootstrap(self.rank, self.world, self.producer_rank, self._fn, None, self.nproducers)
 
 
 def schedule(losses=None, *, s_iter, e_iter, total_infers, t_train, t_infer, t_p=-1.0, t_c=-1.0, s_model=0.0,

@@ -78,6 +78,17 @@ def test_xproc_no_torn_reads(nproc, fanout):
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("nproc,nprod,mode,config", [(3, 2, 0, "ptychonn"), (5, 2, 0, "resnet50"),
+                                                    (5, 3, 1, "small"), (4, 2, 1, "ptychonn")])
+def test_xproc_data_parallel_producers(nproc, nprod, mode, config):
+    """SURVEY s8(f) N1: data-parallel producers each pack their chunk share;
+    consumers assemble every version from all of them."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py", ["--config", config, "--mode", str(mode), "--nprod",
+                                                           str(nprod), "--versions", "5"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 def test_xproc_fault_injection():
     rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fault", "1", "--versions", "3"])
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]

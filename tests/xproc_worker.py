@@ -78,6 +78,7 @@ def main():
     ap.add_argument("--versions", type=int, default=6)
     ap.add_argument("--fault", type=int, default=0)
     ap.add_argument("--stress", type=int, default=0, help="ASYNC publishes while consumers verify every view")
+    ap.add_argument("--nprod", type=int, default=1, help="data-parallel producers (ranks 0..nprod-1)")
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
@@ -87,8 +88,9 @@ def main():
         [(f"t{i}", synth.F32, (1000 + 37 * i,)) for i in range(7)] + [("odd", synth.BYTES, (13,))]
     seed = synth.SEEDS.get(a.config, 0xC0FFEE)
     tensors = G.alloc_model(specs, device=f"cuda:{dev}")
-    bs = V.Bootstrap(rank, world, producer_rank=0)
-    role = V.PRODUCER if rank == 0 else V.CONSUMER
+    bs = V.Bootstrap(rank, world, producer_rank=0, nproducers=a.nprod)
+    is_prod = rank < a.nprod
+    role = V.PRODUCER if is_prod else V.CONSUMER
     m = V.Model(f"xp-{a.config}", role, tensors, tier=a.tier, mode=a.mode, fanout=a.fanout, device=dev,
                 bootstrap=bs)
     errors = 0
@@ -100,7 +102,7 @@ def main():
         if a.fault and rank == 1 and v == 2:
             m.fault_next()
         dist.barrier()
-        if rank == 0:
+        if is_prod:
             G.fill_model(tensors, specs, seed, v)
             torch.cuda.synchronize()
             try:
@@ -115,11 +117,13 @@ def main():
                 seals = V._from_ptr(sp, like).view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2)
                 exp = [synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
                 off, S = T.layout([e.size for e in exp], 256)
-                if not np.array_equal(seals, T.seal(T.pack(exp, off, S), 2 << 20, v)):
-                    print(f"[rank0] seals differ at v{v}", flush=True)
+                ref = T.seal(T.pack(exp, off, S), 2 << 20, v)
+                own = [c for c in range(n) if c % a.nprod == rank]  # data-parallel: this producer's chunks
+                if not np.array_equal(seals[own], ref[own]):
+                    print(f"[rank{rank}] seals differ at v{v}", flush=True)
                     errors += 1
         dist.barrier()
-        if rank != 0 and a.mode == V.SYNC:
+        if not is_prod and a.mode == V.SYNC:
             view = m.acquire_latest(timeout_us=5_000_000)
             want = 1 if (a.fault and rank == 1 and v == 2) else v
             if view.version != want:
@@ -136,7 +140,7 @@ def main():
                     break
             m.release(view)
         dist.barrier()
-    if rank != 0 and a.mode == V.ASYNC and not a.stress:
+    if not is_prod and a.mode == V.ASYNC and not a.stress:
         m.wait_installed(a.versions, timeout_us=20_000_000)
         view = m.acquire_latest()
         if view.version != a.versions:
@@ -149,10 +153,10 @@ def main():
         st = m.stats()
         print(f"[rank{rank}] installs={st['installs']} skipped={st['skipped']}", flush=True)
     dist.barrier()
-    if rank != 0:
+    if not is_prod:
         m.close()
     dist.barrier()
-    if rank == 0:
+    if is_prod:
         m.close()
     t = torch.tensor([errors])
     dist.all_reduce(t)
