@@ -118,11 +118,14 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
     m.nchunks = (uint32_t)((m.s_packed + chunk_bytes - 1) / chunk_bytes);
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    // item size: enough items for ~4 per resident warp, 2 KiB .. 16 KiB, 512-B
-    // multiple.  The 16 KiB cap keeps the fused kernel's read-back window
-    // (resident warps x item) at ~77 MB, inside the 126 MB L2.
+    // item size: enough items for ~4 per resident warp, 2 KiB .. 8 KiB, 512-B
+    // multiple (VIPER_ITEM_MAX / VIPER_ITEM_MIN override, for sweeps).  Small
+    // items keep the fused kernel's read-back L2-resident and balance the tail.
     uint64_t target = m.s_packed / ((uint64_t)sms * 32 * 4) + 1;
-    uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), 16384);
+    uint64_t cap = 8192;  // sweep: profiles/r01/item_sweep.log (best for the fused kernel)
+    if (const char *e = getenv("VIPER_ITEM_MAX")) cap = std::max<uint64_t>(512, strtoull(e, nullptr, 10) / 512 * 512);
+    uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), cap);
+    if (const char *e = getenv("VIPER_ITEM_MIN")) item_max = std::max<uint64_t>(item_max, strtoull(e, nullptr, 10) / 512 * 512);
     if (item_max > chunk_bytes) item_max = chunk_bytes;
     m.items.clear();
     std::vector<uint32_t> per_chunk(m.nchunks, 0);
