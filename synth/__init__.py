@@ -45,6 +45,9 @@ SEEDS = {
     "vit_b16": 0x5EED0003,
     "gpt2_xl": 0x5EED0004,
     "llama3_8b": 0x5EED0005,
+    "nt3a_600mb": 0x5EED0006,
+    "tc1_4p7gb": 0x5EED0007,
+    "ptychonn_4p5gb": 0x5EED0008,
 }
 
 
@@ -199,6 +202,32 @@ def _llama3_8b():
     return out
 
 
+def _paper_sized(total_bytes: int, n_conv: int, dense_in: int):
+    """fp32 parameter set of a given checkpoint size, shaped like the paper's
+    1D-CNN workloads (CANDLE NT3/TC1: a few conv1d kernels, then dense layers
+    holding almost all bytes; PAPER.md s5.2 P:2016-2054, sizes P:2115-2117)."""
+    out = []
+    ch = 1
+    for i in range(n_conv):
+        out.append((f"conv{i}.weight", F32, (128, ch, 20)))
+        out.append((f"conv{i}.bias", F32, (128,)))
+        ch = 128
+    used = sum(nbytes_of(s) for s in out)
+    left = (total_bytes - used) // 4
+    # two dense layers: dense_in -> h (the bulk), h -> 200, then the head
+    h = max(1, (left - 200 * 2 - 2) // (dense_in + 200 + 1))
+    out += [("dense0.weight", F32, (h, dense_in)), ("dense0.bias", F32, (h,)),
+            ("dense1.weight", F32, (200, h)), ("dense1.bias", F32, (200,)),
+            ("head.weight", F32, (2, 200)), ("head.bias", F32, (2,))]
+    return out
+
+
+PAPER_SIZED = {  # PAPER.md P:2115-2117 checkpoint sizes (GB = 1e9 B, reading R18)
+    "nt3a_600mb": lambda: _paper_sized(600_000_000, 2, 60483 * 2),
+    "tc1_4p7gb": lambda: _paper_sized(4_700_000_000, 2, 60483 * 8),
+    "ptychonn_4p5gb": lambda: _paper_sized(4_500_000_000, 4, 65536 * 4),
+}
+
 _RECIPES = {
     "ptychonn": _ptychonn,
     "resnet50": _resnet50,
@@ -213,6 +242,8 @@ CONFIGS = ["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"]
 
 def model_specs(name: str):
     """Ordered [(tensor_name, dtype, shape)] for a workload."""
+    if name in PAPER_SIZED:
+        return list(PAPER_SIZED[name]())
     return list(_RECIPES[name]())
 
 
