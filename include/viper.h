@@ -126,6 +126,12 @@ typedef struct {
     const viper_tensor *slot1; /* consumer: optional caller-owned second replica
                                   (same n, nbytes); NULL -> library allocates it  */
     int32_t flags;           /* VIPER_FLAG_*                                        */
+    const char *flush_dir;   /* producer: background flush of every published version
+                                to <flush_dir>/<model>.v<version>.viper ("all
+                                historical DNN models are flushed ... through a
+                                background thread").  Pinned double
+                                buffer; a version is skipped (counted) when storage
+                                is behind.  NULL = off.  Not with nproducers > 1.  */
 } viper_config;
 
 typedef struct viper_model viper_model; /* opaque */
@@ -225,6 +231,7 @@ typedef struct {
                                   in-process: pack + install + verify + swap in one launch)     */
     int32_t last_status;
     int32_t nconsumers;
+    uint64_t flushed, flush_skipped, flush_last;  /* producer with flush_dir        */
 } viper_stats;
 viper_status viper_get_stats(viper_model *m, viper_stats *out);
 
@@ -239,6 +246,17 @@ viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_s
 /* Test hook (T4 fault injection): the consumer's next install flips one
  * staged bit before verification -> VIPER_E_CHECKSUM, version not installed. */
 viper_status viper_debug_fault_next(viper_model *m);
+
+/*
+ * viper_restore -- read a flushed version back (fault tolerance / resume).
+ * Copies the file's packed snapshot to the GPU and installs it into
+ * `tensors` (device pointers on `device`) with the install kernel, which
+ * re-verifies every item seal: VIPER_E_CHECKSUM if the file was corrupted,
+ * VIPER_E_INVAL if it does not describe these n tensors.  Synchronous on
+ * cuda_stream; *version_out receives the file's version.
+ */
+viper_status viper_restore(const char *path, const viper_tensor *tensors, int32_t n, int32_t device,
+                           void *cuda_stream, uint64_t *version_out);
 
 /* Tear down (joins the update thread, frees library-owned memory). */
 viper_status viper_unregister(viper_model *m);

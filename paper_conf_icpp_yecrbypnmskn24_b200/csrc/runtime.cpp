@@ -102,7 +102,7 @@ viper_status stream_write(cudaStream_t st, void *dev_addr, uint64_t v) {
 // LAY (R16) + the warp work list.  Items never cross a seal chunk
 // and are at most item_max bytes; splits fall on 16-B multiples of the tensor.
 viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes,
-                                   uint32_t align, int device) {
+                                   uint32_t align, int device, uint64_t force_item_max) {
     m.n = n;
     m.nbytes.resize(n);
     m.offsets.resize(n);
@@ -126,7 +126,9 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
     if (const char *e = getenv("VIPER_ITEM_MAX")) cap = std::max<uint64_t>(512, strtoull(e, nullptr, 10) / 512 * 512);
     uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), cap);
     if (const char *e = getenv("VIPER_ITEM_MIN")) item_max = std::max<uint64_t>(item_max, strtoull(e, nullptr, 10) / 512 * 512);
+    if (force_item_max) item_max = force_item_max;  // restore: the partition the seals were made with
     if (item_max > chunk_bytes) item_max = chunk_bytes;
+    m.item_max = item_max;
     m.items.clear();
     std::vector<uint32_t> per_chunk(m.nchunks, 0);
     for (int32_t i = 0; i < n; i++) {
@@ -698,6 +700,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     ra.share_n = (uint32_t)p->nprod;
     ra.share_me = (uint32_t)p->pidx;
     CUDA_TRY(launch_seal_reduce(ra, p->side));
+    if (p->flusher) {  // background flush of this version, off the training stream
+        viper_status s = flush_enqueue(p, v, b);
+        if (s) return s;
+    }
     CUDA_TRY(cudaEventRecord(p->ev_sealed[b], p->side));
     TRACE(4);
     if (sync && dram) launch_all();
@@ -759,6 +765,7 @@ static void free_model(viper_model *m) {
     }
     cudaSetDevice(m->device);
     cudaDeviceSynchronize();
+    flush_stop(m);
     if (m->rec) m->rec->active.store(0);
     if (m->xproc) xproc_free(m);
     if (m->chan) {
@@ -869,7 +876,9 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
             if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
             m->chan->producer = m;
         }
-        return alloc_producer(m, tensors);
+        viper_status ps = alloc_producer(m, tensors);
+        if (ps == VIPER_OK && m->cfg.flush_dir) ps = flush_start(m, m->cfg.flush_dir);
+        return ps;
     }
     if ((st = alloc_consumer(m, tensors))) return st;
     {
@@ -1079,6 +1088,7 @@ viper_status viper_get_stats(viper_model *m, viper_stats *out) {
     std::lock_guard<std::mutex> lk(m->stats_mu);
     *out = m->stats;
     out->nconsumers = m->ctrl ? m->ctrl->ncons.load() : 0;
+    flush_stats(m, &out->flushed, &out->flush_skipped, &out->flush_last);
     return VIPER_OK;
 }
 

@@ -75,6 +75,7 @@ struct Manifest {
     uint32_t align = 0;
     std::vector<BaseItem> items;
     std::vector<uint32_t> chunk_first;  // [nchunks + 1]
+    uint64_t item_max = 0;
     uint32_t nchunks = 0;
     uint32_t *d_chunk_first = nullptr;
     // DRAM-tier pieces: [byte_lo, byte_hi) and [item_lo, item_hi), whole chunks
@@ -83,6 +84,7 @@ struct Manifest {
 };
 
 struct Channel;
+struct Flusher;
 
 // Where a consumer reads snapshot slot b from: the producer's device buffers
 // (same process, or CUDA-IPC peer-mapped over NVLink), the host staging of the
@@ -173,6 +175,7 @@ struct viper_model {
     uint64_t sa_S = 0, sa_IS = 0;
     int32_t rank = 0, world = 1;
     bool early_notify = false;                       // producer: consumers pipeline behind the pack
+    vp::Flusher *flusher = nullptr;                  // producer: background flush (flush.cpp)
     int32_t nprod = 1, pidx = 0;                     // data-parallel producers / this producer's index
     uint32_t pack_nitems = 0;                        // items this producer packs (its chunk share)
     void *peer_snap_m[vp::kMaxProducers] = {};        // consumer: every producer's snapshot (IPC)
@@ -206,7 +209,7 @@ int64_t now_ns();
 void futex_wake_all(std::atomic<uint32_t> *w);
 void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us);
 viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint64_t chunk_bytes, uint32_t align,
-                            int device);
+                            int device, uint64_t force_item_max = 0);
 viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out, uint32_t share_n,
                           uint32_t share_me, uint32_t *count);
 std::atomic<uint64_t> &pub_word(viper_model *p);
@@ -225,6 +228,12 @@ SnapSource source_of(const viper_model *p);
 // stream memory operations (driver entry points, resolved at first use)
 viper_status stream_wait_geq(cudaStream_t st, const void *dev_addr, uint64_t v);
 viper_status stream_write(cudaStream_t st, void *dev_addr, uint64_t v);
+
+// flush.cpp
+viper_status flush_start(viper_model *m, const char *dir);
+viper_status flush_enqueue(viper_model *p, uint64_t v, int b);
+void flush_stop(viper_model *m);
+void flush_stats(viper_model *m, uint64_t *flushed, uint64_t *skipped, uint64_t *last);
 
 // xproc.cpp
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);

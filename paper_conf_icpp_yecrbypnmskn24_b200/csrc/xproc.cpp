@@ -235,8 +235,11 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
     const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
     const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
     const size_t ctrl_bytes = page_up(sizeof(Ctrl));
+    if (st == VIPER_OK && producer && m->cfg.flush_dir && M > 1)
+        st = set_error(VIPER_E_UNSUPPORTED, "flush with data-parallel producers");
     if (st == VIPER_OK && producer) {
         st = alloc_producer(m, tensors);
+        if (st == VIPER_OK && m->cfg.flush_dir) st = flush_start(m, m->cfg.flush_dir);
         const size_t bytes = ctrl_bytes + (dram ? 2 * (S + IS) : 0);
         if (st == VIPER_OK && m->pidx == 0) st = create_segment(m, bytes, me.shm_path, sizeof me.shm_path);
         if (st == VIPER_OK && m->pidx == 0) {

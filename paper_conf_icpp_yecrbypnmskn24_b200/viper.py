@@ -42,7 +42,7 @@ class viper_bootstrap(C.Structure):
 class viper_config(C.Structure):
     _fields_ = [("tier", C.c_int32), ("fanout", C.c_int32), ("mode", C.c_int32), ("chunk_bytes", C.c_uint64),
                 ("align", C.c_uint32), ("device", C.c_int32), ("slot1", C.POINTER(viper_tensor)),
-                ("flags", C.c_int32)]
+                ("flags", C.c_int32), ("flush_dir", C.c_char_p)]
 
 
 class viper_view(C.Structure):
@@ -55,7 +55,8 @@ class viper_stats(C.Structure):
                 ("installs", C.c_uint64), ("skipped", C.c_uint64), ("failures", C.c_uint64),
                 ("t_publish_us", C.c_double), ("t_install_us", C.c_double), ("t_notify_us", C.c_double),
                 ("writer_wait_us", C.c_double), ("t_pack_dev_us", C.c_double),
-                ("t_install_dev_us", C.c_double), ("t_fused_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32)]
+                ("t_install_dev_us", C.c_double), ("t_fused_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32),
+                ("flushed", C.c_uint64), ("flush_skipped", C.c_uint64), ("flush_last", C.c_uint64)]
 
 
 class viper_sched_in(C.Structure):
@@ -78,7 +79,7 @@ UPDATE_CB = C.CFUNCTYPE(None, C.c_uint64, C.c_int32, C.c_void_p)
 # every symbol include/viper.h declares (checked by tests/test_abi.py)
 EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_acquire_latest", "viper_release",
            "viper_wait_installed", "viper_get_stats", "viper_layout", "viper_debug_buffers", "viper_debug_fault_next", "viper_unregister",
-           "viper_schedule", "viper_strerror", "viper_last_error", "viper_version"]
+           "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version"]
 
 _lib = None
 _lock = threading.Lock()
@@ -117,6 +118,8 @@ def lib() -> C.CDLL:
             L.viper_debug_fault_next.argtypes = [C.c_void_p]
             L.viper_unregister.argtypes = [C.c_void_p]
             L.viper_schedule.argtypes = [C.POINTER(viper_sched_in), C.POINTER(viper_sched_out)]
+            L.viper_restore.argtypes = [C.c_char_p, C.POINTER(viper_tensor), C.c_int32, C.c_int32, C.c_void_p,
+                                        C.POINTER(C.c_uint64)]
             L.viper_strerror.argtypes = [C.c_int32]
             L.viper_strerror.restype = C.c_char_p
             L.viper_last_error.restype = C.c_char_p
@@ -188,14 +191,16 @@ class Model:
     """One endpoint (producer or consumer) of a model-update channel."""
 
     def __init__(self, name: str, role: int, tensors, *, tier=TIER_GPU, fanout=FANOUT_DIRECT, mode=SYNC,
-                 chunk_bytes=0, align=0, device=None, slot1=None, flags=0, bootstrap=None, names=None):
+                 chunk_bytes=0, align=0, device=None, slot1=None, flags=0, bootstrap=None, names=None,
+                 flush_dir=None):
         L = lib()
         self.tensors = list(tensors)
         self.role = role
         if device is None:
             device = self.tensors[0].device.index if self.tensors and self.tensors[0].is_cuda else 0
         descs, self._keep = _tensor_descs(self.tensors, names)
-        cfg = viper_config(tier, fanout, mode, chunk_bytes, align, device, None, flags)
+        self._flush_dir = flush_dir.encode() if flush_dir else None
+        cfg = viper_config(tier, fanout, mode, chunk_bytes, align, device, None, flags, self._flush_dir)
         if slot1 is not None:
             s1, k1 = _tensor_descs(slot1, names)
             self._keep += [s1, k1]
@@ -300,6 +305,17 @@ class Bootstrap:
     def struct(self) -> viper_bootstrap:
         self._fn = ALLGATHER_FN(self._allgather)
         return viper_bootstrap(self.rank, self.world, self.producer_rank, self._fn, None, self.nproducers)
+
+
+def restore(path: str, tensors, device=None, stream=None) -> int:
+    """Install a flushed version (viper_restore) into `tensors`; returns its version."""
+    if device is None:
+        device = tensors[0].device.index if tensors and tensors[0].is_cuda else 0
+    descs, keep = _tensor_descs(list(tensors))
+    v = C.c_uint64(0)
+    check(lib().viper_restore(path.encode(), descs, len(tensors), device, _stream_ptr(stream), C.byref(v)),
+          f"viper_restore({path})")
+    return int(v.value)
 
 
 def schedule(losses=None, *, s_iter, e_iter, total_infers, t_train, t_infer, t_p=-1.0, t_c=-1.0, s_model=0.0,
