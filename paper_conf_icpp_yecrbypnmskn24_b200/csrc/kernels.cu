@@ -402,10 +402,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fus
         const uint64_t part = warp_sum(copy_item_fused((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
                                                        a.ncons, it.nbytes, it.packed_off, lane, inject, got));
         const uint64_t sealed = part + a.version * kVerMix;
-        __syncwarp();
-        if (lane == 0) {
+        if (lane == 0) {  // no concurrent reader in this path: a plain store (grid end publishes it)
             a.iseal[w].mixed = sealed;
-            st_release(&a.iseal[w].version, a.version);
+            a.iseal[w].version = a.version;
         }
 #pragma unroll
         for (int k = 0; k < kMaxFused; k++) {
@@ -619,6 +618,8 @@ cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
     pack_seal_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
+
+const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
 
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
     publish_fused_kernel<<<g.grid, g.block, 0, st>>>(a);

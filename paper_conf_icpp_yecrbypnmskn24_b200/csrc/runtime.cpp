@@ -509,6 +509,29 @@ viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
 int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug_trace)
 #define TRACE(i) (g_trace[i] = now_ns())
 
+// The fused kernel through a one-node CUDA graph whose parameters are updated
+// per publish: measured cheaper on the host than a direct launch
+// (profiles/r01/launchcal.log).  VIPER_NO_GRAPH=1 launches directly.
+static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStream_t st) {
+    static const bool no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));
+    if (no_graph) return launch_fused(f, p->geo, st);
+    void *args[] = {(void *)&f};
+    cudaKernelNodeParams kp{};
+    kp.func = (void *)fused_kernel_fn();
+    kp.gridDim = dim3(p->geo.grid);
+    kp.blockDim = dim3(p->geo.block);
+    kp.kernelParams = args;
+    cudaError_t e;
+    if (!p->fused_exec) {
+        if ((e = cudaGraphCreate(&p->fused_graph, 0)) != cudaSuccess) return e;
+        if ((e = cudaGraphAddKernelNode(&p->fused_node, p->fused_graph, nullptr, 0, &kp)) != cudaSuccess) return e;
+        if ((e = cudaGraphInstantiate(&p->fused_exec, p->fused_graph, 0)) != cudaSuccess) return e;
+    } else if ((e = cudaGraphExecKernelNodeSetParams(p->fused_exec, p->fused_node, &kp)) != cudaSuccess) {
+        return e;
+    }
+    return cudaGraphLaunch(p->fused_exec, st);
+}
+
 std::atomic<uint64_t> &pub_word(viper_model *p) {
     return p->nprod > 1 ? p->ctrl->pub_m[p->pidx] : p->ctrl->pub_state;
 }
@@ -611,7 +634,9 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
             prepared[k].c->stats.writer_wait_us = prepared[k].waited_us;
         }
         if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
-        CUDA_TRY(launch_fused(f, p->geo, st));
+        TRACE(8);
+        CUDA_TRY(launch_fused_fast(p, f, st));
+        TRACE(9);
         if (timing) {
             CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
             p->timing_pending = true;
@@ -790,6 +815,8 @@ static void free_model(viper_model *m) {
         for (int k = 0; k < 2; k++)
             if (evs[k]) cudaEventDestroy(evs[k]);
     if (m->ev_packed) cudaEventDestroy(m->ev_packed);
+    if (m->fused_exec) cudaGraphExecDestroy(m->fused_exec);
+    if (m->fused_graph) cudaGraphDestroy(m->fused_graph);
     if (m->side) cudaStreamDestroy(m->side);
     if (m->ustream) cudaStreamDestroy(m->ustream);
     delete m;

@@ -130,6 +130,9 @@ struct viper_model {
     cudaEvent_t ev_t[2] = {nullptr, nullptr};        // VIPER_FLAG_TIMING: around the kernel
     bool timing_pending = false;
     bool last_fused = false;                         // last publish used publish_fused_kernel
+    cudaGraph_t fused_graph = nullptr;               // one-node graph: cheaper per-publish launch
+    cudaGraphExec_t fused_exec = nullptr;
+    cudaGraphNode_t fused_node = nullptr;
     cudaStream_t side = nullptr;                     // DRAM-tier D2H stream
     uint8_t *h_stage[2] = {nullptr, nullptr};        // DRAM tier (pinned)
     vp::ISeal *h_iseal[2] = {nullptr, nullptr};

@@ -131,6 +131,7 @@ cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
 cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device);
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
+const void *fused_kernel_fn();  // for the one-node launch graph (runtime.cpp)
 // pdl: the install directly follows the pack on `st` (programmatic dependent launch)
 cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl);
 

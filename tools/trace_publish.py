@@ -28,9 +28,9 @@ for v in range(1, 60):
     t1 = time.monotonic_ns()
     L.viper_debug_trace(buf, 16)
     if v > 10:
-        rows.append([buf[i] - buf[0] for i in range(8)] + [buf[0] - t0, t1 - buf[7]])
+        rows.append([buf[i] - buf[0] for i in range(8)] + [buf[0] - t0, t1 - buf[7], buf[8] - buf[0], buf[9] - buf[0]])
 names = ["entry", "pinscan", "installs_prepared", "pack+install_launched", "reduce+events", "status_seen", "finish", "exit",
-         "py->C", "C->py"]
+         "py->C", "C->py", "before_fused_launch", "after_fused_launch"]
 for i, n in enumerate(names):
     print(f"{n:18s} {statistics.median(r[i] for r in rows) / 1e3:8.2f} us")
 c.close()
