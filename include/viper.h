@@ -258,6 +258,18 @@ viper_status viper_debug_fault_next(viper_model *m);
 viper_status viper_restore(const char *path, const viper_tensor *tensors, int32_t n, int32_t device,
                            void *cuda_stream, uint64_t *version_out);
 
+/* Test hooks: the CUDA-free version protocol (protocol.h) over a POSIX shm
+ * segment of `words` u64 per slot, for multi-process CPU tests.  publish(v)
+ * fills snapshot slot v&1 after it is unpinned; install pins the latest
+ * snapshot and swaps it into consumer cidx's double buffer; read acquires a
+ * slot and counts words != its version (torn reads), then releases it. */
+viper_status viper_debug_proto_create(const char *path, uint64_t words, int32_t ncons, void **out);
+viper_status viper_debug_proto_open(const char *path, uint64_t words, void **out);
+viper_status viper_debug_proto_close(void *h, int32_t unlink_it, const char *path);
+viper_status viper_debug_proto_publish(void *h, uint64_t v);
+viper_status viper_debug_proto_install(void *h, int32_t cidx, uint64_t *installed, uint64_t *torn_snapshot);
+viper_status viper_debug_proto_read(void *h, int32_t cidx, uint64_t *version, uint64_t *torn);
+
 /* Tear down (joins the update thread, frees library-owned memory). */
 viper_status viper_unregister(viper_model *m);
 

@@ -1,0 +1,68 @@
+// protocol.h -- the host-side version protocol (SURVEY s8(a) a3/a7/a8,
+// DESIGN.md s7), free of CUDA so that it is exercised by CPU multi-process
+// tests (selftest.cpp) exactly as the engine uses it.
+//
+//   producer slot reuse  pub_state <- newer; fence; scan pins   (wait_unpinned)
+//   consumer snapshot pin pin <- v; fence; re-read pub_state     (pin_latest)
+//   writer (install)     wait ref[target] == 0                   (wait_readers_gone)
+//   reader               s <- state; ref[slot]++; re-read state  (try_acquire_slot)
+// All seq_cst std::atomic on words that may live in a shared-memory segment.
+#pragma once
+#include <sched.h>
+
+#include <atomic>
+#include <cstdint>
+
+#include "runtime.h"
+
+namespace vp {
+
+// Producer: before overwriting the snapshot slot that holds old_v, wait until
+// no active consumer pins old_v.  Returns false (and *who) on timeout.
+inline bool wait_unpinned(Ctrl *ctrl, uint64_t old_v, int64_t timeout_ns, int *who) {
+    const int nc = ctrl->ncons.load();
+    for (int i = 0; i < nc; i++) {
+        const int64_t w0 = now_ns();
+        while (ctrl->cons[i].active.load() && ctrl->cons[i].pin.load() == old_v) {
+            if (now_ns() - w0 > timeout_ns) {
+                if (who) *who = i;
+                return false;
+            }
+            __builtin_ia32_pause();
+        }
+    }
+    return true;
+}
+
+// Writer: the alternative copy is written only once no reader pins it.
+inline bool wait_readers_gone(ConsRec *r, int target, int64_t timeout_ns) {
+    const int64_t t0 = now_ns();
+    while (r->ref[target].load() != 0) {
+        if (now_ns() - t0 > timeout_ns) return false;
+        sched_yield();
+    }
+    return true;
+}
+
+// Reader: pin the active slot; returns the state word (version << 1 | slot)
+// with ref[slot] held, or 0 when nothing >= min_version is installed.
+inline uint64_t try_acquire_slot(ConsRec *r, uint64_t min_version) {
+    for (;;) {
+        const uint64_t s = r->state.load();
+        if (s == 0 || (s >> 1) < min_version) return 0;
+        const int slot = (int)(s & 1);
+        r->ref[slot].fetch_add(1);
+        if (r->state.load() == s) return s;
+        r->ref[slot].fetch_sub(1);  // swapped under us: retry
+    }
+}
+
+inline void release_slot(ConsRec *r, int slot) { r->ref[slot].fetch_sub(1); }
+
+// The slot an install writes: the inactive one (slot 0 before the first install).
+inline int install_target(ConsRec *r) {
+    const uint64_t cur = r->state.load();
+    return cur == 0 ? 0 : (int)(1 - (cur & 1));
+}
+
+}  // namespace vp

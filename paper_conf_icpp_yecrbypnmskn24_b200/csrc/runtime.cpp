@@ -7,6 +7,7 @@
 // Every byte moves in the kernels of kernels.cu; this file only decides what
 // to launch, when, and on which stream.  There is no CPU data path.
 #include "runtime.h"
+#include "protocol.h"
 
 #include <cuda.h>  // types of the driver entry points (no libcuda link)
 #include <linux/futex.h>
@@ -290,14 +291,10 @@ bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
 // and build the kernel arguments.  Caller holds c->install_mu.
 viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, int b, PreparedInstall *pi) {
     ConsRec *r = c->rec;
-    const uint64_t cur = r->state.load();
-    const int target = cur == 0 ? 0 : (int)(1 - (cur & 1));
+    const int target = install_target(r);
     const int64_t t0 = now_ns();
-    while (r->ref[target].load() != 0) {
-        if (now_ns() - t0 > 10ll * 1000000000ll)
-            return set_error(VIPER_E_TIMEOUT, "readers kept slot %d pinned for 10 s", target);
-        sched_yield();
-    }
+    if (!wait_readers_gone(r, target, 10ll * 1000000000ll))
+        return set_error(VIPER_E_TIMEOUT, "readers kept slot %d pinned for 10 s", target);
     pi->c = c;
     pi->waited_us = (now_ns() - t0) / 1e3;
     InstallArgs &a = pi->a;
@@ -558,16 +555,9 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     // buffer).  pub_state already names a newer version, so late
     // pinners of old_v fail their re-validation.
     if (old_v) {
-        const int nc = ctrl->ncons.load();
-        for (int i = 0; i < nc; i++) {
-            const int64_t w0 = now_ns();
-            while (ctrl->cons[i].active.load() && ctrl->cons[i].pin.load() == old_v) {
-                if (now_ns() - w0 > 10ll * 1000000000ll)
-                    return set_error(VIPER_E_TIMEOUT, "consumer %d kept snapshot v%llu pinned", i,
-                                     (unsigned long long)old_v);
-                cpu_relax();
-            }
-        }
+        int who = -1;
+        if (!wait_unpinned(ctrl, old_v, 10ll * 1000000000ll, &who))
+            return set_error(VIPER_E_TIMEOUT, "consumer %d kept snapshot v%llu pinned", who, (unsigned long long)old_v);
         // the DRAM-tier D2H of old_v must be finished before overwriting
         if (p->cfg.tier == VIPER_TIER_DRAM) CUDA_TRY(cudaStreamWaitEvent(st, p->ev_ready[b], 0));
         // ... and so must the side-stream seal reduction reading its item seals
@@ -1028,20 +1018,19 @@ viper_status viper_acquire_latest(viper_model *m, uint64_t min_version, int64_t 
             r->waiters.fetch_sub(1);
             continue;
         }
-        const int slot = (int)(s & 1);
-        r->ref[slot].fetch_add(1);
-        if (r->state.load() == s) {
+        const uint64_t got = try_acquire_slot(r, min_version);
+        if (got) {
+            const int slot = (int)(got & 1);
             std::lock_guard<std::mutex> lk(m->views_mu);
             const uint64_t t = m->next_ticket++;
             m->views[t] = ViewTicket{slot};
-            out->version = s >> 1;
+            out->version = got >> 1;
             out->slot = slot;
             out->ntensors = m->man.n;
             out->dev_ptrs = m->slot_ptrs[slot].data();
             out->ticket = t;
             return VIPER_OK;
         }
-        r->ref[slot].fetch_sub(1);  // swapped under us: retry
     }
 }
 

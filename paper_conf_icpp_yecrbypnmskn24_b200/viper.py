@@ -79,7 +79,9 @@ UPDATE_CB = C.CFUNCTYPE(None, C.c_uint64, C.c_int32, C.c_void_p)
 # every symbol include/viper.h declares (checked by tests/test_abi.py)
 EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_acquire_latest", "viper_release",
            "viper_wait_installed", "viper_get_stats", "viper_layout", "viper_debug_buffers", "viper_debug_fault_next", "viper_unregister",
-           "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version"]
+           "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version",
+           "viper_debug_proto_create", "viper_debug_proto_open", "viper_debug_proto_close",
+           "viper_debug_proto_publish", "viper_debug_proto_install", "viper_debug_proto_read"]
 
 _lib = None
 _lock = threading.Lock()
@@ -118,6 +120,13 @@ def lib() -> C.CDLL:
             L.viper_debug_fault_next.argtypes = [C.c_void_p]
             L.viper_unregister.argtypes = [C.c_void_p]
             L.viper_schedule.argtypes = [C.POINTER(viper_sched_in), C.POINTER(viper_sched_out)]
+            L.viper_debug_proto_create.argtypes = [C.c_char_p, C.c_uint64, C.c_int32, C.POINTER(C.c_void_p)]
+            L.viper_debug_proto_open.argtypes = [C.c_char_p, C.c_uint64, C.POINTER(C.c_void_p)]
+            L.viper_debug_proto_close.argtypes = [C.c_void_p, C.c_int32, C.c_char_p]
+            L.viper_debug_proto_publish.argtypes = [C.c_void_p, C.c_uint64]
+            L.viper_debug_proto_install.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_uint64),
+                                                    C.POINTER(C.c_uint64)]
+            L.viper_debug_proto_read.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]
             L.viper_restore.argtypes = [C.c_char_p, C.POINTER(viper_tensor), C.c_int32, C.c_int32, C.c_void_p,
                                         C.POINTER(C.c_uint64)]
             L.viper_strerror.argtypes = [C.c_int32]

@@ -97,3 +97,10 @@ def test_xproc_fault_injection():
 def test_bootstrap_allgather_gloo_world2():
     rc, out = run_torchrun(2, "tests/bootstrap_worker.py", [], timeout=120)
     assert rc == 0 and "BOOTSTRAP_OK" in out, out[-3000:]
+
+
+def test_protocol_two_processes_gloo_cpu():
+    """The cross-process version protocol on a real shm segment, CPU only:
+    0 torn snapshot copies, 0 torn reads, no version regress over 3000 publishes."""
+    rc, out = run_torchrun(2, "tests/protocol_worker.py", [], timeout=180)
+    assert rc == 0 and "PROTO_RESULT errors=0" in out, out[-3000:]
