@@ -177,7 +177,8 @@ def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
     """Same update through the public API with HOST buffers: the trainer's
     parameters live in one flat device buffer (tensor views at 256-B aligned
     offsets); each step copies the new weights from a flat pinned host buffer
-    (one H2D), publishes, and reads the seal digest back (D2H)."""
+    (one cudaMemcpyAsync H2D), publishes, and reads the chunk-seal digest of
+    the installed version back (D2H)."""
     import torch
     specs = synth.model_specs(name)
     seed = synth.SEEDS[name]
@@ -193,13 +194,15 @@ def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
     host = []
     for i in range(2):  # two host versions of the whole flat buffer, alternated
         G.fill_model(prod_t, specs, seed, 1000 + i)
-        host.append(flat.cpu().pin_memory())
+        hb = G.PinnedBuffer(flat.numel())
+        hb.view()[:] = flat.cpu().numpy()
+        host.append(hb)
     mname = f"e2e-{name}-{os.getpid()}-{time.monotonic_ns()}"
     cons = V.Model(mname, V.CONSUMER, cons_t)
     prod = V.Model(mname, V.PRODUCER, prod_t)
     st = torch.cuda.current_stream()
-    _, seals_ptr, nchunks = prod.debug_buffers()
-    digest = torch.empty(2 * nchunks, dtype=torch.int64).pin_memory()
+    _, _, nchunks = prod.debug_buffers()
+    digest = G.PinnedBuffer(16 * nchunks)
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     times = []
     try:
@@ -207,52 +210,23 @@ def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
             G.l2_flush(flush_buf, stream=st)
             torch.cuda.synchronize()
             ev0.record(st)
-            flat.copy_(host[i % 2], non_blocking=True)
+            host[i % 2].to_device(flat, stream=st)
             prod.publish(i + 1, stream=st)
             _, seals_ptr, _ = prod.debug_buffers()
-            like = torch.empty(4 * nchunks, dtype=torch.int32, device="cuda")
-            digest.copy_(V._from_ptr(seals_ptr, like).view(torch.int64), non_blocking=True)
+            digest.from_device_ptr(seals_ptr, 16 * nchunks, stream=st)
             ev1.record(st)
             ev1.synchronize()
             if i >= warmup:
                 times.append(ev0.elapsed_time(ev1))
-        ok = digest.numel() == 2 * nchunks
+        d = digest.view().view("<u8").reshape(nchunks, 2)
+        ok = bool((d[:, 0] == warmup + steps).all())
     finally:
         cons.close()
         prod.close()
-    return {"ms": statistics.mean(times), "h2d": flat.numel(), "d2h": digest.numel() * 8, "ok": ok}
-
-
-def c5_schedule(V, G, synth, flush, gpu_row):
-    """BASELINE.json configs[4]: Llama-3 8B through the pinned-DRAM tier vs the
-    GPU tier (1-GPU loopback here), each driving viper_schedule (the paper's
-    IPP, s4.3) with the engine's measured costs: t_p = producer stall (the
-    pack for the GPU tier; pack + host copy for DRAM), t_c =
-    consumer load (the install / H2D + install), on a synthetic Exp3 warm-up
-    loss curve with the paper's Fig. 6 time magnitudes."""
-    import numpy as np
-    d = run_update_bench(V, G, synth, "llama3_8b", 3, 2, flush, tier=V.TIER_DRAM)
-    dram_ms = statistics.mean(d["dev_ms"])
-    gpu_ms = gpu_row.get("latency_ms")
-    rng = np.random.default_rng(5)
-    x = np.arange(50.0)
-    warm = list(2.5 * np.exp(-0.02 * x) + 0.8 + rng.normal(0, 0.01, 50))
-    t_train, t_infer = 0.07, 0.006
-    s_iter, e_iter = 50, 2000
-    total = int((e_iter - s_iter) * t_train / t_infer)
-    res = {"dram_update_ms": round(dram_ms, 3), "gpu_update_ms": gpu_ms,
-           "dram_over_gpu": round(dram_ms / gpu_ms, 2) if gpu_ms else None,
-           "paper_context": "TC1 Host-Async / GPU-Async latency 2.326 s / 0.856 s = 2.7x (Polaris, inter-node)"}
-    for tier, t_p, t_c in (("gpu", gpu_row.get("pack_us", 0) * 1e-6, gpu_row.get("install_us", 0) * 1e-6),
-                           ("dram", dram_ms * 1e-3 / 2, dram_ms * 1e-3 / 2)):
-        sch = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
-                         t_p=t_p, t_c=t_c, x=list(x))
-        gr = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
-                        t_p=t_p, t_c=t_c, x=list(x), algo=V.SCHED_GREEDY)
-        res[tier] = {"t_p_s": t_p, "t_c_s": t_c, "family": ["Exp2", "Exp3", "Lin2", "Expd3"][sch["family"]],
-                     "fixed_interval": sch["best_interval"], "fixed_cil": round(sch["predicted_cil"], 3),
-                     "greedy_checkpoints": len(gr["sched"]), "greedy_cil": round(gr["predicted_cil"], 3)}
-    return res
+        for hb in host:
+            hb.close()
+        digest.close()
+    return {"ms": statistics.mean(times), "h2d": flat.numel(), "d2h": 16 * nchunks, "ok": ok}
 
 
 def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
@@ -568,7 +542,7 @@ def gpu_arm(args):
     if rank == 0:
         e = run_e2e(V, G, synth, name, max(3, args.steps // 2), args.warmup, flush)
         out["e2e"] = {"value": round(e["ms"], 6), "unit": "ms", "h2d_bytes_per_step": e["h2d"],
-                      "d2h_bytes_per_step": e["d2h"]}
+                      "d2h_bytes_per_step": e["d2h"], "digest_ok": e["ok"]}
         if not args.no_sweep:
             sweep = {}
             for nm in ["resnet50", "vit_b16", "gpt2_xl", "llama3_8b"]:

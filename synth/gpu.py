@@ -21,6 +21,11 @@ def lib():
         _lib.l2_flush.restype = C.c_int
         _lib.launch_empty.argtypes = [C.c_void_p]
         _lib.launch_empty.restype = C.c_int
+        _lib.host_alloc.argtypes = [C.c_uint64]
+        _lib.host_alloc.restype = C.c_void_p
+        _lib.host_free.argtypes = [C.c_void_p]
+        _lib.copy_async.argtypes = [C.c_void_p, C.c_void_p, C.c_uint64, C.c_int, C.c_void_p]
+        _lib.copy_async.restype = C.c_int
     return _lib
 
 
@@ -57,3 +62,33 @@ def l2_flush(buf, stream=None):
 def empty_kernel(stream=None):
     if lib().launch_empty(_sp(stream)) != 0:
         raise RuntimeError("launch_empty failed")
+
+
+H2D, D2H = 1, 2
+
+
+class PinnedBuffer:
+    """cudaHostAlloc'ed host buffer (bench e2e leg) with raw async copies."""
+
+    def __init__(self, nbytes: int):
+        self.nbytes = nbytes
+        self.ptr = lib().host_alloc(max(nbytes, 1))
+        if not self.ptr:
+            raise MemoryError("cudaHostAlloc failed")
+
+    def view(self):
+        import numpy as np
+        return np.ctypeslib.as_array((C.c_uint8 * max(self.nbytes, 1)).from_address(self.ptr))[: self.nbytes]
+
+    def to_device(self, dev_tensor, stream=None):
+        if lib().copy_async(C.c_void_p(dev_tensor.data_ptr()), C.c_void_p(self.ptr), self.nbytes, H2D, _sp(stream)):
+            raise RuntimeError("H2D failed")
+
+    def from_device_ptr(self, dev_ptr: int, nbytes: int, stream=None):
+        if lib().copy_async(C.c_void_p(self.ptr), C.c_void_p(dev_ptr), nbytes, D2H, _sp(stream)):
+            raise RuntimeError("D2H failed")
+
+    def close(self):
+        if self.ptr:
+            lib().host_free(C.c_void_p(self.ptr))
+            self.ptr = None

@@ -72,3 +72,15 @@ extern "C" int launch_empty(void *stream) {
 extern "C" int l2_flush(void *dev_ptr, uint64_t bytes, void *stream) {
     return cudaMemsetAsync(dev_ptr, (int)(bytes & 0xFF), bytes, (cudaStream_t)stream) == cudaSuccess ? 0 : -3;
 }
+
+// Harness helpers for bench.py's e2e leg: pinned host buffers and copies
+// through the CUDA runtime directly (torch's pinned copy path measured
+// erratic H2D throughput on this VM, profiles/r01/h2dcal.log).
+extern "C" void *host_alloc(uint64_t bytes) {
+    void *p = nullptr;
+    return cudaHostAlloc(&p, bytes, cudaHostAllocPortable) == cudaSuccess ? p : nullptr;
+}
+extern "C" int host_free(void *p) { return cudaFreeHost(p) == cudaSuccess ? 0 : -3; }
+extern "C" int copy_async(void *dst, const void *src, uint64_t bytes, int kind, void *stream) {
+    return cudaMemcpyAsync(dst, src, bytes, (cudaMemcpyKind)kind, (cudaStream_t)stream) == cudaSuccess ? 0 : -3;
+}
