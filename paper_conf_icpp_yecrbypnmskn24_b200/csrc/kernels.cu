@@ -34,6 +34,9 @@ namespace {
 #ifndef VP_UNROLL
 #define VP_UNROLL 8
 #endif
+#ifndef VP_FUSED_PREFETCH
+#define VP_FUSED_PREFETCH 0  // A/B: no measurable gain (profiles/r01/ktime_prefetch_ab.log)
+#endif
 constexpr int kWarpsPerBlock = VP_WARPS_PER_BLOCK;  // 256 threads
 constexpr int kBlocksPerSM = VP_BLOCKS_PER_SM;      // 512 threads / SM resident (128-reg budget)
 constexpr int kUnroll = VP_UNROLL;                  // 16-B vectors in flight per lane per step
@@ -231,8 +234,12 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
     asm volatile("griddepcontrol.launch_dependents;");
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
-    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
-        const Item it = a.items[w];
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    Item nxt{};
+    if (w < a.nitems) nxt = a.items[w];
+    for (; w < a.nitems; w += nwarps) {
+        const Item it = nxt;  // descriptor prefetched one item ahead: its load overlaps this item's stream
+        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
         const uint64_t part = warp_sum(copy_item<false>((const uint8_t *)it.ptr, a.packed + it.packed_off,
                                                         it.nbytes, it.packed_off, lane, false));
         __syncwarp();  // every lane's stores are ordered before lane 0's release
@@ -389,8 +396,18 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fus
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
-    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+#if VP_FUSED_PREFETCH
+    Item nxt{};
+    if (w < a.nitems) nxt = a.items[w];
+#endif
+    for (; w < a.nitems; w += nwarps) {
+#if VP_FUSED_PREFETCH
+        const Item it = nxt;  // descriptor prefetched one item ahead
+        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
+#else
         const Item it = a.items[w];
+#endif
         uint64_t cptr[kMaxFused];  // only the slot address differs between the lists
         uint32_t inject = 0;
 #pragma unroll

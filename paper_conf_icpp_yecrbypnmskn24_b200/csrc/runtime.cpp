@@ -122,7 +122,8 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
     // item size: enough items for ~4 per resident warp, 2 KiB .. 8 KiB, 512-B
     // multiple (VIPER_ITEM_MAX / VIPER_ITEM_MIN override, for sweeps).  Small
     // items keep the fused kernel's read-back L2-resident and balance the tail.
-    uint64_t target = m.s_packed / ((uint64_t)sms * 32 * 4) + 1;
+    // ~4 items per resident warp (16 warps / SM: kernels.cu geometry)
+    uint64_t target = m.s_packed / ((uint64_t)sms * 16 * 4) + 1;
     uint64_t cap = 8192;  // sweep: profiles/r01/item_sweep.log (best for the fused kernel)
     if (const char *e = getenv("VIPER_ITEM_MAX")) cap = std::max<uint64_t>(512, strtoull(e, nullptr, 10) / 512 * 512);
     uint64_t item_max = std::min<uint64_t>(std::max<uint64_t>((target + 511) / 512 * 512, 2048), cap);
