@@ -107,7 +107,7 @@ enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install
                                     times appear in viper_stats (bench.py)       */
        VIPER_FLAG_NO_FUSE = 4,   /* producer: never use the fused SYNC kernel
                                     (pack and install as separate kernels)      */
-       VIPER_FLAG_TMA = 8,       /* producer: pack through TMA bulk copies
+       VIPER_FLAG_TMA = 8,       /* producer pack / consumer install: TMA bulk copies
                                     (cp.async.bulk global<->shared) instead of
                                     128-bit register streaming; implies NO_FUSE.
                                     Without the flag the TMA pack is picked

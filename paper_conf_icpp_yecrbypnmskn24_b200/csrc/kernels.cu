@@ -269,6 +269,28 @@ __global__ void seal_reduce_kernel(const SealReduceArgs a) {
     }
 }
 
+// End of an install grid: the last block to finish publishes the result and,
+// when every item matched, swaps the version word from the device.
+__device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
+    if (bad) atomicOr(a.err, kErrChecksum);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();  // cumulative over the block's stores (ordered by the barrier)
+        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
+            __threadfence();
+            const uint32_t e = atomicExch(a.err, 0u);
+            *a.done = 0;
+            const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
+            // Every block's slot stores are GPU-visible (cumulative fences
+            // above); later readers are kernels launched after the host saw
+            // the flip, so plain system-visible stores suffice here.
+            if (a.status_h) *a.status_h = st;
+            if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
+            if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
+        }
+    }
+}
+
 // install: stream every item packed -> slot tensor, recompute its seal and
 // compare with the producer's; the last block to finish publishes the result
 // and, if every item matched, swaps the version word from the device.
@@ -369,23 +391,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
         }
     }
-    if (bad) atomicOr(a.err, kErrChecksum);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();  // cumulative over the block's stores (ordered by the barrier)
-        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
-            __threadfence();
-            const uint32_t e = atomicExch(a.err, 0u);
-            *a.done = 0;
-            const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
-            // Every block's slot stores are GPU-visible (cumulative fences
-            // above); later readers are kernels launched after the host saw
-            // the flip, so plain system-visible stores suffice here.
-            if (a.status_h) *a.status_h = st;
-            if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
-            if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
-        }
-    }
+    install_finish(a, bad);
 }
 
 // SYNC in-process publish, pack + install fused per warp.  Lane l re-reads
@@ -599,6 +605,110 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const 
     (void)issued;
 }
 
+// install_verify, TMA bulk-copy variant (direct installs not PDL-chained to
+// their pack: ASYNC, DRAM tier, cross-process).  Snapshot pieces stream
+// through the same per-warp shared-memory ring: cp.async.bulk global ->
+// shared, checksum from shared memory, cp.async.bulk shared -> slot tensor.
+// The grid's last block swaps the version once every bulk store completed.
+__global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(const InstallArgs a) {
+    extern __shared__ __align__(128) uint8_t tma_smem[];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    uint8_t *stage = tma_smem + wib * (kTmaStages * kTmaStage);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(tma_smem + kTmaWarps * kTmaStages * kTmaStage) + wib * kTmaStages;
+    if (lane == 0) {
+        for (int s = 0; s < kTmaStages; s++) mbar_init(bar + s);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    const uint32_t nwarps = gridDim.x * kTmaWarps;
+    const uint32_t w0 = blockIdx.x * kTmaWarps + wib;
+    auto body_of = [&](const Item &it) -> uint32_t {
+        return ((it.ptr | it.packed_off) & 15u) ? 0u : (it.nbytes & ~15u);
+    };
+    TmaCursor ld{w0, 0};
+    auto next_piece = [&](TmaCursor &c, Item &it, uint32_t &bytes) -> bool {
+        while (c.w < a.nitems) {
+            it = a.items[c.w];
+            const uint32_t body = body_of(it);
+            if (c.off < body) {
+                bytes = min(kTmaStage, body - c.off);
+                return true;
+            }
+            c.w += nwarps;
+            c.off = 0;
+        }
+        return false;
+    };
+    for (int s = 0; s < kTmaStages; s++) {  // prologue: fill the ring
+        Item it;
+        uint32_t bytes;
+        if (!next_piece(ld, it, bytes)) break;
+        if (lane == 0) {
+            mbar_expect_tx(bar + s, bytes);
+            bulk_g2s(stage + s * kTmaStage, a.packed + it.packed_off + ld.off, bytes, bar + s);
+        }
+        ld.off += bytes;
+    }
+    uint32_t consumed = 0, phase_bits = 0;
+    bool bad = false;
+    for (uint32_t w = w0; w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        uint64_t expect = 0;
+        if (lane == 0) {  // not PDL-chained: the seal is already there; still never hang
+            const ISeal *is = a.iseal + w;
+            uint64_t waited = 0;
+            while (ld_acquire_sys(&is->version) != a.version) {
+                __nanosleep(256);
+                if ((waited += 256) > kItemWaitNs) {
+                    atomicOr(a.err, kErrTimeout);
+                    break;
+                }
+            }
+            expect = is->mixed;
+        }
+        const uint32_t body = body_of(it);
+        uint64_t acc = 0;
+        for (uint32_t off = 0; off < body; off += kTmaStage) {
+            const uint32_t bytes = min(kTmaStage, body - off);
+            const int s = consumed % kTmaStages;
+            mbar_wait(bar + s, (phase_bits >> s) & 1u);
+            phase_bits ^= 1u << s;
+            uint8_t *buf = stage + s * kTmaStage;
+            if (w == a.fault_item && off == 0 && lane == 0) buf[0] ^= 0x10;  // fault injection (tests)
+            __syncwarp();
+            const uint32_t g0 = (uint32_t)((it.packed_off + off) >> 2);
+            for (uint32_t i = lane; i < bytes / 16; i += 32)
+                acc += cks_vec(*reinterpret_cast<const uint4 *>(buf + i * 16), g0 + 4u * i);
+            __syncwarp();
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                bulk_s2g((uint8_t *)it.ptr + off, buf, bytes);
+            }
+            consumed++;
+            Item nit;
+            uint32_t nbytes;
+            if (next_piece(ld, nit, nbytes)) {
+                if (lane == 0) {
+                    bulk_wait_read<0>();
+                    mbar_expect_tx(bar + s, nbytes);
+                    bulk_g2s(stage + s * kTmaStage, a.packed + nit.packed_off + ld.off, nbytes, bar + s);
+                }
+                ld.off += nbytes;
+            }
+        }
+        if (body < it.nbytes)
+            acc += (body == 0) ? copy_item<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes, it.packed_off,
+                                                 lane, w == a.fault_item)
+                               : copy_words_bytewise<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, body,
+                                                           it.nbytes, it.packed_off, lane, false);
+        const uint64_t part = warp_sum(acc);
+        if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // slot stores complete
+    __syncwarp();
+    install_finish(a, bad);
+}
+
 }  // namespace
 
 Geometry pick_geometry(uint32_t nitems, int device) {
@@ -640,6 +750,22 @@ const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
 
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
     publish_fused_kernel<<<g.grid, g.block, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device) {
+    static int sms = 0;
+    const size_t smem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
+    if (sms == 0) {
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) sms = 148;
+        cudaError_t e =
+            cudaFuncSetAttribute(install_verify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    const uint32_t want = (a.nitems + kTmaWarps - 1) / kTmaWarps;
+    const uint32_t cap = (uint32_t)sms * 2;
+    const int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+    install_verify_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
     return cudaGetLastError();
 }
 

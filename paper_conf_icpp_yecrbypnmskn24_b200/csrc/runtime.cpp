@@ -342,8 +342,16 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     }
     c->rec->status.store(1);  // "in flight"
     const bool timing = c->cfg.flags & VIPER_FLAG_TIMING;
+    // TMA bulk-copy install: direct pulls whose snapshot is complete before the
+    // kernel starts (not PDL-chained, no early notification), forced by
+    // VIPER_FLAG_TMA or auto up to 1 GiB like the pack
+    const bool direct = pi.a.sa_n == 0 && pi.a.mp_n <= 1;
+    const bool complete = !(pdl && !timing) && !c->ctrl->early_notify.load();
+    const bool tma = direct && complete && !(c->cfg.flags & VIPER_FLAG_NO_TMA) &&
+                     ((c->cfg.flags & VIPER_FLAG_TMA) || c->man.s_packed <= (1ull << 30));
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
-    CUDA_TRY(launch_install(pi.a, c->geo, st, pdl && !timing));
+    if (tma) CUDA_TRY(launch_install_tma(pi.a, st, c->device));
+    else CUDA_TRY(launch_install(pi.a, c->geo, st, pdl && !timing));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
         c->timing_pending = true;

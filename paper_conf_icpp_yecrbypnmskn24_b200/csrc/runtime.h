@@ -60,6 +60,7 @@ struct alignas(64) Ctrl {
     // every producer published it
     alignas(64) std::atomic<uint64_t> pub_m[kMaxProducers];
     std::atomic<int32_t> nprod;
+    std::atomic<int32_t> early_notify;   // producer names v before its pack completed
 };
 
 // Pointer-free work item (the device lists add each endpoint's tensor address).

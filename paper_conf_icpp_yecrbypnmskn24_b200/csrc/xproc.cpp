@@ -305,6 +305,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (all[r].role != VIPER_PRODUCER && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
         const char *env = getenv("VIPER_EARLY_NOTIFY");
         m->early_notify = env ? atoi(env) != 0 : other;
+        if (m->pidx == 0) m->ctrl->early_notify.store(m->early_notify ? 1 : 0);
     }
     if (st == VIPER_OK && !producer) {
         int idx = 0;
