@@ -309,6 +309,38 @@ def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
             "pickup_note": "publish -> update-thread pickup, includes waiting for the previous install"}
 
 
+def c5_schedule(V, G, synth, flush, gpu_row):
+    """BASELINE.json configs[4]: Llama-3 8B through the pinned-DRAM tier vs the
+    GPU tier (1-GPU loopback here), each driving viper_schedule (the paper's
+    IPP, s4.3) with the engine's measured costs: t_p = producer stall (the
+    pack for the GPU tier; pack + host copy for DRAM), t_c =
+    consumer load (the install / H2D + install), on a synthetic Exp3 warm-up
+    loss curve with the paper's Fig. 6 time magnitudes."""
+    import numpy as np
+    d = run_update_bench(V, G, synth, "llama3_8b", 3, 2, flush, tier=V.TIER_DRAM)
+    dram_ms = statistics.mean(d["dev_ms"])
+    gpu_ms = gpu_row.get("latency_ms")
+    rng = np.random.default_rng(5)
+    x = np.arange(50.0)
+    warm = list(2.5 * np.exp(-0.02 * x) + 0.8 + rng.normal(0, 0.01, 50))
+    t_train, t_infer = 0.07, 0.006
+    s_iter, e_iter = 50, 2000
+    total = int((e_iter - s_iter) * t_train / t_infer)
+    res = {"dram_update_ms": round(dram_ms, 3), "gpu_update_ms": gpu_ms,
+           "dram_over_gpu": round(dram_ms / gpu_ms, 2) if gpu_ms else None,
+           "paper_context": "TC1 Host-Async / GPU-Async latency 2.326 s / 0.856 s = 2.7x (Polaris, inter-node)"}
+    for tier, t_p, t_c in (("gpu", gpu_row.get("pack_us", 0) * 1e-6, gpu_row.get("install_us", 0) * 1e-6),
+                           ("dram", dram_ms * 1e-3 / 2, dram_ms * 1e-3 / 2)):
+        sch = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
+                         t_p=t_p, t_c=t_c, x=list(x))
+        gr = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
+                        t_p=t_p, t_c=t_c, x=list(x), algo=V.SCHED_GREEDY)
+        res[tier] = {"t_p_s": t_p, "t_c_s": t_c, "family": ["Exp2", "Exp3", "Lin2", "Expd3"][sch["family"]],
+                     "fixed_interval": sch["best_interval"], "fixed_cil": round(sch["predicted_cil"], 3),
+                     "greedy_checkpoints": len(gr["sched"]), "greedy_cil": round(gr["predicted_cil"], 3)}
+    return res
+
+
 def event_floor_us(G, reps=20):
     """An empty kernel bracketed exactly like the library's timing events."""
     import torch
@@ -325,7 +357,7 @@ def event_floor_us(G, reps=20):
     return statistics.median(out)
 
 
-def cpu_baseline(synth, name, budget_s=10.0, max_updates=400):
+def cpu_baseline(synth, name, budget_s=10.0, max_updates=100000):
     """The oracle (plain C, single thread, as it stands) timed on this host's
     cores on a bounded sample: repeated updates of the same config."""
     from oracle import transfer as T
