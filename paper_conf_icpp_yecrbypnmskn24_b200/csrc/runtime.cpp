@@ -222,6 +222,12 @@ static viper_status channel_open(const std::string &name, const Manifest &man, C
     return VIPER_OK;
 }
 
+static viper_model *channel_producer(Channel *ch) {
+    if (!ch) return nullptr;
+    std::lock_guard<std::mutex> lk(ch->pmu);
+    return ch->producer;
+}
+
 static void channel_close(Channel *ch) {
     std::lock_guard<std::mutex> lk(g_reg_mu);
     if (--ch->refs > 0) return;
@@ -427,7 +433,7 @@ void update_loop(viper_model *c) {
             if (c->xproc) {  // cross-process: this thread installs every version it sees
                 work = ps != 0 && (ps >> 1) > c->attempted;
             } else {
-                viper_model *p = c->chan ? c->chan->producer : nullptr;
+                viper_model *p = channel_producer(c->chan);
                 const bool async = p && p->cfg.mode == VIPER_ASYNC;
                 work = p && ps != 0 && (ps >> 1) > c->attempted && (async || c->attempted == 0);
             }
@@ -465,7 +471,9 @@ void update_loop(viper_model *c) {
         if (c->xproc) {
             st = xproc_install(c, v, b);
         } else {
-            viper_model *p = c->chan ? c->chan->producer : nullptr;
+            // install_mu is held through the stream sync below: a producer
+            // teardown drains this before freeing the buffers read here
+            viper_model *p = channel_producer(c->chan);
             st = p ? enqueue_install(c, source_of(p), v, b, c->ustream, true)
                    : set_error(VIPER_E_STATE, "producer gone");
         }
@@ -584,12 +592,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     std::vector<std::unique_lock<std::mutex>> locks;
     std::vector<PreparedInstall> prepared;
     const SnapSource psrc = source_of(p);
+    std::unique_lock<std::mutex> chan_lock;
     if (sync && p->chan) {
-        std::vector<viper_model *> cons;
-        {
-            std::lock_guard<std::mutex> lk(g_reg_mu);
-            cons = p->chan->consumers;
-        }
+        chan_lock = std::unique_lock<std::mutex>(p->chan->mu);  // consumers stay registered until we return
+        const std::vector<viper_model *> cons = p->chan->consumers;
         for (viper_model *c : cons) {
             std::unique_lock<std::mutex> lk(c->install_mu);
             if (c->attempted >= v) continue;
@@ -787,20 +793,31 @@ static void free_model(viper_model *m) {
         }
         m->upd.join();
     }
+    if (m->chan) {
+        Channel *ch = m->chan;
+        if (m->role == VIPER_PRODUCER) {
+            {
+                std::lock_guard<std::mutex> lk(ch->pmu);
+                if (ch->producer == m) ch->producer = nullptr;
+            }
+            // drain installs that may still read this producer's buffers; the
+            // consumers cannot disappear meanwhile: their teardown takes ch->mu
+            std::lock_guard<std::mutex> lk(ch->mu);
+            for (viper_model *c : ch->consumers) {
+                std::lock_guard<std::mutex> il(c->install_mu);
+            }
+        } else {
+            std::lock_guard<std::mutex> lk(ch->mu);  // waits for an in-flight SYNC publish
+            auto &v = ch->consumers;
+            v.erase(std::remove(v.begin(), v.end(), m), v.end());
+        }
+    }
     cudaSetDevice(m->device);
     cudaDeviceSynchronize();
     flush_stop(m);
     if (m->rec) m->rec->active.store(0);
     if (m->xproc) xproc_free(m);
-    if (m->chan) {
-        {
-            std::lock_guard<std::mutex> lk(g_reg_mu);
-            auto &v = m->chan->consumers;
-            v.erase(std::remove(v.begin(), v.end(), m), v.end());
-            if (m->chan->producer == m) m->chan->producer = nullptr;
-        }
-        channel_close(m->chan);
-    }
+    if (m->chan) channel_close(m->chan);
     cudaFree(m->man.d_chunk_first);
     cudaFree(m->d_items);
     cudaFree(m->d_slot_items[0]);
@@ -897,18 +914,17 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
     m->ctrl = m->chan->ctrl;
     m->ctrl_dev = m->chan->ctrl_dev;
     if (m->role == VIPER_PRODUCER) {
-        {
-            std::lock_guard<std::mutex> lk(g_reg_mu);
-            if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
-            m->chan->producer = m;
-        }
         viper_status ps = alloc_producer(m, tensors);
         if (ps == VIPER_OK && m->cfg.flush_dir) ps = flush_start(m, m->cfg.flush_dir);
-        return ps;
+        if (ps) return ps;
+        std::lock_guard<std::mutex> lk(m->chan->pmu);  // visible only once fully built
+        if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
+        m->chan->producer = m;
+        return VIPER_OK;
     }
     if ((st = alloc_consumer(m, tensors))) return st;
     {
-        std::lock_guard<std::mutex> lk(g_reg_mu);
+        std::lock_guard<std::mutex> lk(m->chan->mu);
         const int idx = m->ctrl->ncons.load();
         if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
         m->cidx = idx;

@@ -192,9 +192,16 @@ struct viper_model {
 
 namespace vp {
 
+// Locking (in-process channel):
+//   mu   guards `consumers`; a SYNC publish holds it for its whole duration, so
+//        a consumer cannot be torn down while the producer installs into it.
+//   pmu  leaf lock for `producer`; update threads read it while holding their
+//        own install_mu, so a producer teardown that nulls it and then cycles
+//        every consumer's install_mu knows no install still uses its buffers.
 struct Channel {
     std::string name;
     Ctrl *ctrl = nullptr, *ctrl_dev = nullptr;
+    std::mutex mu, pmu;
     viper_model *producer = nullptr;
     std::vector<viper_model *> consumers;
     int refs = 0;

@@ -386,3 +386,34 @@ def test_full_size_loopback_sampled(name, flags):
     finally:
         close_all(prod, cons)
         torch.cuda.empty_cache()
+
+
+def test_teardown_races_in_process():
+    """Unregistering a producer while its consumers' update threads install
+    (ASYNC), and consumers while publishes run, never crashes or hangs."""
+    specs = [(f"t{i}", synth.F32, (200_000,)) for i in range(4)]
+    for rep in range(5):
+        prod, prod_t, cons, cons_t = make_pair(specs, 1, ncons=3, mode=V.ASYNC)
+        stop = threading.Event()
+
+        def publisher():
+            v = 0
+            while not stop.is_set():
+                v += 1
+                try:
+                    prod.publish(v)
+                except V.ViperError:
+                    break
+
+        th = threading.Thread(target=publisher)
+        th.start()
+        time.sleep(0.01)
+        cons[rep % 3].close()          # a consumer leaves mid-stream
+        time.sleep(0.01)
+        stop.set()
+        th.join()
+        prod.close()                   # producer leaves while others may install
+        time.sleep(0.005)
+        for i, c in enumerate(cons):
+            if i != rep % 3:
+                c.close()
