@@ -34,12 +34,20 @@ namespace {
 #ifndef VP_UNROLL
 #define VP_UNROLL 8
 #endif
+#ifndef VP_FUSED_UNROLL
+#define VP_FUSED_UNROLL 8
+#endif
+#ifndef VP_FUSED_BLOCKS
+#define VP_FUSED_BLOCKS 2
+#endif
 #ifndef VP_FUSED_PREFETCH
 #define VP_FUSED_PREFETCH 0  // A/B: no measurable gain (profiles/r01/ktime_prefetch_ab.log)
 #endif
 constexpr int kWarpsPerBlock = VP_WARPS_PER_BLOCK;  // 256 threads
 constexpr int kBlocksPerSM = VP_BLOCKS_PER_SM;      // 512 threads / SM resident (128-reg budget)
 constexpr int kUnroll = VP_UNROLL;                  // 16-B vectors in flight per lane per step
+constexpr int kFusedUnroll = VP_FUSED_UNROLL;       // publish_fused_kernel's own geometry
+constexpr int kFusedBlocks = VP_FUSED_BLOCKS;
 
 __device__ __forceinline__ uint4 ld_stream(const void *p) {
     uint4 r;
@@ -159,6 +167,7 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
 // (same lane, same addresses -> ordered; an L2 hit), and store them into each
 // consumer's slot.  Returns the pack checksum; cks_c[k] is the checksum of
 // what consumer k received (the read-back, after any injected fault).
+template <int U = kUnroll>
 __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ src, uint8_t *__restrict__ snap,
                                                     const uint64_t *dst, uint32_t ncons, uint32_t n, uint64_t p0,
                                                     uint32_t lane, uint32_t inject_mask, uint64_t *cks_c) {
@@ -178,15 +187,15 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
     }
     const uint32_t nvec = n >> 4;
     const uint32_t g0 = (uint32_t)(p0 >> 2);
-    for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
-        uint4 r[kUnroll];
+    for (uint32_t base = 0; base < nvec; base += 32 * U) {
+        uint4 r[U];
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
+        for (int u = 0; u < U; u++) {
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) r[u] = ld_stream(src + (size_t)i * 16);
         }
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
+        for (int u = 0; u < U; u++) {
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) {
                 st_v4(snap + (size_t)i * 16, r[u]);
@@ -194,7 +203,7 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
             }
         }
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {  // read back what this lane stored
+        for (int u = 0; u < U; u++) {  // read back what this lane stored
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) r[u] = ld_cg(snap + (size_t)i * 16);
         }
@@ -202,7 +211,7 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
         for (int k = 0; k < kMaxFused; k++) {
             if (k >= (int)ncons) break;
 #pragma unroll
-            for (int u = 0; u < kUnroll; u++) {
+            for (int u = 0; u < U; u++) {
                 const uint32_t i = base + u * 32 + lane;
                 if (i < nvec) {
                     uint4 x = r[u];
@@ -398,7 +407,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
 // exactly the snapshot bytes it stored (same thread, so ordered) with L2
 // loads, installs them and recomputes the item checksum; the seal check is
 // against the value just sealed.  No cross-warp dependency inside the grid.
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fused_kernel(const FusedArgs a) {
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fused_kernel(const FusedArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
@@ -422,7 +431,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) publish_fus
             if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
         }
         uint64_t got[kMaxFused] = {0, 0, 0, 0};
-        const uint64_t part = warp_sum(copy_item_fused((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
+        const uint64_t part = warp_sum(copy_item_fused<kFusedUnroll>((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
                                                        a.ncons, it.nbytes, it.packed_off, lane, inject, got));
         const uint64_t sealed = part + a.version * kVerMix;
         if (lane == 0) {  // no concurrent reader in this path: a plain store (grid end publishes it)
@@ -717,6 +726,7 @@ Geometry pick_geometry(uint32_t nitems, int device) {
         if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) sms = 148;
     }
     Geometry g;
+    g.items = nitems;
     g.block = kWarpsPerBlock * 32;
     const uint32_t want = (nitems + kWarpsPerBlock - 1) / kWarpsPerBlock;
     const uint32_t cap = (uint32_t)sms * kBlocksPerSM;
@@ -747,6 +757,17 @@ cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
 }
 
 const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
+
+Geometry fused_geometry(const Geometry &g) {
+    // same block shape, up to kFusedBlocks resident blocks per SM
+    Geometry f = g;
+    static int sms = 0;
+    if (sms == 0 && (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0) != cudaSuccess || sms <= 0)) sms = 148;
+    const int cap = sms * kFusedBlocks;
+    const int want = (int)((g.items + kWarpsPerBlock - 1) / kWarpsPerBlock);
+    f.grid = want < 1 ? 1 : (want > cap ? cap : want);
+    return f;
+}
 
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
     publish_fused_kernel<<<g.grid, g.block, 0, st>>>(a);

@@ -528,12 +528,13 @@ int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug
 // (profiles/r01/launchcal.log).  VIPER_NO_GRAPH=1 launches directly.
 static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStream_t st) {
     static const bool no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));
-    if (no_graph) return launch_fused(f, p->geo, st);
+    const Geometry fg = fused_geometry(p->geo);
+    if (no_graph) return launch_fused(f, fg, st);
     void *args[] = {(void *)&f};
     cudaKernelNodeParams kp{};
     kp.func = (void *)fused_kernel_fn();
-    kp.gridDim = dim3(p->geo.grid);
-    kp.blockDim = dim3(p->geo.block);
+    kp.gridDim = dim3(fg.grid);
+    kp.blockDim = dim3(fg.block);
     kp.kernelParams = args;
     cudaError_t e;
     if (!p->fused_exec) {

@@ -123,7 +123,9 @@ struct FusedArgs {
 
 struct Geometry {
     int grid, block;
+    uint32_t items = 0;
 };
+Geometry fused_geometry(const Geometry &g);  // publish_fused_kernel's grid (own occupancy)
 Geometry pick_geometry(uint32_t nitems, int device);
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);

@@ -369,7 +369,9 @@ def test_full_size_loopback_sampled(name, flags):
         seals = _raw_u64(sp, 2 * n).cpu().numpy().view(np.uint64).reshape(n, 2)
         assert np.all(seals[:, 0] == 2)
         rng = np.random.default_rng(0)
-        for c in sorted({0, n - 1, *rng.integers(0, n, 4).tolist()}):
+        # every chunk seal where the oracle finishes in seconds, else a sample
+        every = S <= 256 << 20
+        for c in (range(n) if every else sorted({0, n - 1, *rng.integers(0, n, 4).tolist()})):
             assert int(seals[c, 1]) == T.expected_chunk_seal(specs, seed, 2, offsets, S, 2 << 20, c), c
         view = cons[0].acquire_latest()
         assert view.version == 2
