@@ -101,20 +101,21 @@ enum { VIPER_SYNC = 0,   /* publish returns after every consumer installed v (or
        VIPER_ASYNC = 1 };/* publish returns once the snapshot is enqueued on cuda_stream;
                             delivery and install proceed in the background       */
 
-/* Debug flags (viper_config.flags). */
-enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install
-                                    kernels on their launch streams; the device
-                                    times appear in viper_stats (bench.py)       */
-       VIPER_FLAG_NO_FUSE = 4,   /* producer: never use the fused SYNC kernel
-                                    (pack and install as separate kernels)      */
-       VIPER_FLAG_TMA = 8,       /* producer pack / consumer install: TMA bulk copies
-                                    (cp.async.bulk global<->shared) instead of
-                                    128-bit register streaming; implies NO_FUSE.
-                                    Without the flag the TMA pack is picked
-                                    automatically for packs not PDL-chained to an
-                                    install (ASYNC, DRAM tier, cross-process) of
-                                    models <= 1 GiB, where it measured faster  */
-       VIPER_FLAG_NO_TMA = 16 }; /* producer: never auto-select the TMA pack     */
+/* Flags (viper_config.flags). */
+enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install /
+                                   fused kernels on their launch streams; the
+                                   device times appear in viper_stats (bench.py) */
+       VIPER_FLAG_NO_FUSE = 4,  /* producer: never use the fused SYNC kernel
+                                   (pack and install as separate kernels)        */
+       VIPER_FLAG_TMA = 8,      /* producer: pack with TMA bulk copies (implies
+                                   NO_FUSE); consumer: install with TMA bulk copies
+                                   (cp.async.bulk global<->shared) instead of 128-bit
+                                   register streaming.  Without the flag TMA is
+                                   picked automatically for models <= 1 GiB where it
+                                   applies: packs no install is PDL-chained to
+                                   (ASYNC, DRAM tier, cross-process) and direct
+                                   installs of a completed snapshot               */
+       VIPER_FLAG_NO_TMA = 16 }; /* never auto-select the TMA kernels             */
 
 typedef struct {
     int32_t tier;            /* VIPER_TIER_*                       (default GPU)    */
