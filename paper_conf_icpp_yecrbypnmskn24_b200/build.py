@@ -69,6 +69,22 @@ def build_viper(force: bool = False, verbose: bool = False, out: str = None, def
     return target
 
 
+def build_fast(force: bool = False) -> str:
+    """CPython shim for the per-update calls (publish / acquire / release)."""
+    import sysconfig
+    src = os.path.join(CSRC, "pyfast.c")
+    out = os.path.join(PKG, "_fast" + sysconfig.get_config_var("EXT_SUFFIX"))
+    if not force and not _stale(out, [src]):
+        return out
+    tmp = out + f".tmp{os.getpid()}"
+    cmd = ["gcc", "-O2", "-shared", "-fPIC", "-I", sysconfig.get_paths()["include"], src, "-o", tmp, "-ldl"]
+    r = subprocess.run(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)
+    if r.returncode != 0:
+        raise RuntimeError("pyfast build failed:\n" + r.stdout.decode())
+    os.replace(tmp, out)
+    return out
+
+
 def build_vgen(force: bool = False) -> str:
     if not force and not _stale(VGEN_LIB, [VGEN_SRC]):
         return VGEN_LIB
@@ -82,7 +98,7 @@ def build_vgen(force: bool = False) -> str:
 
 
 def build_all(force: bool = False, verbose: bool = False):
-    return build_viper(force, verbose), build_vgen(force)
+    return build_viper(force, verbose), build_vgen(force), build_fast(force)
 
 
 if __name__ == "__main__":

@@ -85,6 +85,7 @@ EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_ac
 
 _lib = None
 _lock = threading.Lock()
+_fast = None  # CPython shim for publish / acquire / release (csrc/pyfast.c), same libviper.so symbols
 
 
 class ViperError(RuntimeError):
@@ -137,6 +138,13 @@ def lib() -> C.CDLL:
                 fn = getattr(L, f)
                 if fn.restype is C.c_int:  # default
                     fn.restype = C.c_int32
+            global _fast
+            try:
+                from . import _fast as F
+                F.init(LIB_PATH)
+                _fast = F
+            except ImportError:
+                _fast = None
             _lib = L
     return _lib
 
@@ -226,7 +234,13 @@ class Model:
 
     # -- producer
     def publish(self, version: int, stream=None):
-        check(lib().viper_publish(self.h, version, _stream_ptr(stream)), f"viper_publish({version})")
+        if _fast is not None:
+            st = _fast.publish(self.h.value, version, None if stream is None else
+                               (stream if isinstance(stream, int) else stream.cuda_stream))
+        else:
+            st = lib().viper_publish(self.h, version, _stream_ptr(stream))
+        if st:
+            raise ViperError(st, f"viper_publish({version})")
 
     # -- consumer
     def subscribe(self, fn):
@@ -234,11 +248,25 @@ class Model:
         check(lib().viper_subscribe(self.h, self._cb, None), "viper_subscribe")
 
     def acquire_latest(self, min_version=0, timeout_us=0) -> View:
+        if _fast is not None:
+            st, ver, slot, nt, ptrs, ticket = _fast.acquire(self.h.value, min_version, timeout_us)
+            if st:
+                raise ViperError(st, "viper_acquire_latest")
+            v = viper_view(ver, slot, nt, C.cast(C.c_void_p(ptrs), C.POINTER(C.c_void_p)), ticket)
+            return View(self, v)
         v = viper_view()
         check(lib().viper_acquire_latest(self.h, min_version, timeout_us, C.byref(v)), "viper_acquire_latest")
         return View(self, v)
 
     def release(self, view: View, stream=None):
+        if _fast is not None:
+            r = view.raw
+            st = _fast.release(self.h.value, r.version, r.slot, r.ntensors,
+                               C.cast(r.dev_ptrs, C.c_void_p).value or 0, r.ticket,
+                               None if stream is None else (stream if isinstance(stream, int) else stream.cuda_stream))
+            if st:
+                raise ViperError(st, "viper_release")
+            return
         check(lib().viper_release(self.h, C.byref(view.raw), _stream_ptr(stream)), "viper_release")
 
     def wait_installed(self, version: int, timeout_us: int = 10_000_000):
