@@ -10,6 +10,7 @@
 #include "protocol.h"
 
 #include <cuda.h>  // types of the driver entry points (no libcuda link)
+#include <nvtx3/nvToolsExt.h>  // header-only; ranges cost nothing unless a tool attaches
 #include <linux/futex.h>
 #include <sched.h>
 #include <sys/syscall.h>
@@ -68,6 +69,33 @@ void futex_wait(std::atomic<uint32_t> *w, uint32_t expected, int64_t timeout_us)
 }
 
 static inline void cpu_relax() { __builtin_ia32_pause(); }
+
+// NVTX range per stage (publish / install), visible in nsys and usable as an
+// ncu --nvtx filter.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
+// Optional per-update JSON lines (SURVEY s5 metrics): VIPER_LOG=<path>.
+static FILE *g_log = nullptr;
+static std::mutex g_log_mu;
+static std::once_flag g_log_once;
+
+static void log_update(const char *role, const viper_model *m, uint64_t v, viper_status st, double host_us,
+                       double extra_us, const char *extra_name) {
+    std::call_once(g_log_once, [] {
+        if (const char *p = getenv("VIPER_LOG")) g_log = fopen(p, "a");
+    });
+    if (!g_log) return;
+    std::lock_guard<std::mutex> lk(g_log_mu);
+    fprintf(g_log,
+            "{\"t_ns\":%lld,\"role\":\"%s\",\"model\":\"%s\",\"version\":%llu,\"status\":%d,"
+            "\"bytes\":%llu,\"tier\":%d,\"fanout\":%d,\"mode\":%d,\"host_us\":%.3f,\"%s\":%.3f}\n",
+            (long long)now_ns(), role, m->name.c_str(), (unsigned long long)v, st,
+            (unsigned long long)m->man.s_packed, m->cfg.tier, m->cfg.fanout, m->cfg.mode, host_us, extra_name, extra_us);
+    fflush(g_log);
+}
 
 typedef CUresult (*PFN_wait64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
 typedef CUresult (*PFN_write64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
@@ -411,6 +439,7 @@ viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
     }
     r->pin.store(0);
     r->last_status.store(st);
+    log_update("consumer", c, v, st, t_install_us, c->stats.writer_wait_us, "writer_wait_us");
     r->done_version.store(v);
     r->done_seq.fetch_add(1);
     if (r->waiters.load() > 0) futex_wake_all(&r->done_seq);
@@ -467,6 +496,7 @@ void update_loop(viper_model *c) {
         c->attempted = v;
         const int64_t tp = ctrl->pub_time_ns.load();
         const int64_t t0 = now_ns();
+        NvtxRange nvtx("viper_install");
         viper_status st;
         if (c->xproc) {
             st = xproc_install(c, v, b);
@@ -552,6 +582,7 @@ std::atomic<uint64_t> &pub_word(viper_model *p) {
 }
 
 static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st) {
+    NvtxRange nvtx("viper_publish");
     const int64_t t0 = now_ns();
     g_trace[0] = t0;
     if (v == 0 || v <= p->last_version)
@@ -770,6 +801,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         p->stats.last_status = result;
     }
     TRACE(7);
+    log_update("producer", p, v, result, (now_ns() - t0) / 1e3, p->last_fused ? 1.0 : 0.0, "fused");
     return result;
 }
 

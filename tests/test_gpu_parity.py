@@ -2,6 +2,7 @@
 element on the same seeded VGEN inputs, plus the protocol invariants
  on the device path.  Bit-exact throughout: this is
 byte work."""
+import os
 import threading
 import time
 
@@ -419,3 +420,26 @@ def test_teardown_races_in_process():
         for i, c in enumerate(cons):
             if i != rep % 3:
                 c.close()
+
+
+def test_update_log_jsonl(tmp_path):
+    """VIPER_LOG: one JSON line per publish / install (SURVEY s5 metrics)."""
+    import json
+    import subprocess
+    import sys
+    log = tmp_path / "viper.jsonl"
+    code = (
+        "import sys; sys.path.insert(0, '.');"
+        "import synth; from synth import gpu as G; from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V;"
+        "s=synth.model_specs('ptychonn'); pt,ct=G.alloc_model(s),G.alloc_model(s);"
+        "c=V.Model('lg',V.CONSUMER,ct); p=V.Model('lg',V.PRODUCER,pt);"
+        "[p.publish(v) for v in (1,2,3)]; c.close(); p.close()")
+    env = dict(os.environ, VIPER_LOG=str(log))
+    r = subprocess.run([sys.executable, "-c", code], cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                       env=env, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True, timeout=120)
+    assert r.returncode == 0, r.stdout[-2000:]
+    rows = [json.loads(l) for l in log.read_text().splitlines()]
+    prod = [x for x in rows if x["role"] == "producer"]
+    cons = [x for x in rows if x["role"] == "consumer"]
+    assert [x["version"] for x in prod] == [1, 2, 3] and all(x["status"] == 0 for x in rows)
+    assert [x["version"] for x in cons] == [1, 2, 3] and prod[0]["bytes"] == 4618496
