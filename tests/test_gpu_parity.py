@@ -443,3 +443,66 @@ def test_update_log_jsonl(tmp_path):
     cons = [x for x in rows if x["role"] == "consumer"]
     assert [x["version"] for x in prod] == [1, 2, 3] and all(x["status"] == 0 for x in rows)
     assert [x["version"] for x in cons] == [1, 2, 3] and prod[0]["bytes"] == 4618496
+
+
+def test_beyond_16_gib_word_index_wraps():
+    """S > 16 GiB: the CKS word index g is taken mod 2^32 (R16); the
+    chunks straddling g = 2^32 must match the oracle bit for bit."""
+    specs = [("a", synth.BF16, (9 << 29,)), ("b", synth.BF16, (15 << 28,)), ("c", synth.F32, (12345,))]  # 16.5 GiB
+    seed = 0xB16
+    prod, prod_t, cons, cons_t = make_pair(specs, seed)
+    try:
+        G.fill_model(prod_t, specs, seed, 1)
+        prod.publish(1)
+        S, offsets = prod.layout()
+        assert S > (16 << 30)
+        p, sp, n = prod.debug_buffers()
+        seals = _raw_u64(sp, 2 * n).cpu().numpy().view(np.uint64).reshape(n, 2)
+        wrap = (16 << 30) // (2 << 20)  # first chunk whose words have g >= 2^32
+        for c in (0, wrap - 1, wrap, wrap + 1, n - 1):
+            assert int(seals[c, 1]) == T.expected_chunk_seal(specs, seed, 1, offsets, S, 2 << 20, c), c
+        view = cons[0].acquire_latest()
+        for g, pt in zip(view.tensors(cons_t[0]), prod_t):
+            assert torch.equal(g.view(torch.uint8), pt.view(torch.uint8))
+        cons[0].release(view)
+    finally:
+        close_all(prod, cons)
+        del prod_t, cons_t
+        torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_randomized_configurations(seed):
+    """Random tensor lists x {SYNC, ASYNC} x {GPU, DRAM} x {fused, separate,
+    TMA} x {1..5 consumers} x chunk/align choices: every consumer ends
+    byte-identical to VGEN(last version)."""
+    rng = np.random.default_rng(1000 + seed)
+    specs = []
+    for i in range(int(rng.integers(1, 25))):
+        dt = int(rng.choice([synth.F32, synth.BF16, synth.F16, synth.BYTES]))
+        ne = int(rng.choice([0, 1, 5, 4097, int(rng.integers(1, 300_000))]))
+        specs.append((f"t{i}", dt, (ne,)))
+    mode = int(rng.choice([V.SYNC, V.ASYNC]))
+    tier = int(rng.choice([V.TIER_GPU, V.TIER_DRAM]))
+    flags = int(rng.choice([0, V.FLAG_NO_FUSE, V.FLAG_TMA, V.FLAG_NO_TMA]))
+    chunk = int(rng.choice([4096, 65536, 2 << 20]))
+    align = int(rng.choice([16, 256]))
+    ncons = int(rng.integers(1, 6))
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=ncons, mode=mode, tier=tier, flags=flags,
+                                           chunk_bytes=chunk, align=align)
+    try:
+        last = int(rng.integers(2, 6))
+        for v in range(1, last + 1):
+            G.fill_model(prod_t, specs, 7 * seed, v)
+            prod.publish(v)
+        for c, ct in zip(cons, cons_t):
+            c.wait_installed(last, timeout_us=20_000_000)
+            view = c.acquire_latest()
+            assert view.version == last
+            check_slot(view, ct, specs, 7 * seed, last)
+            c.release(view)
+        p_dev, s_dev = device_packed_and_seals(prod)
+        p_or, s_or, _ = oracle_packed_and_seals(specs, 7 * seed, last, chunk, align)
+        assert np.array_equal(p_dev, p_or) and np.array_equal(s_dev, s_or)
+    finally:
+        close_all(prod, cons)
