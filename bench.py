@@ -341,6 +341,31 @@ def c5_schedule(V, G, synth, flush, gpu_row):
     return res
 
 
+def torch_copy_baseline(G, synth, name, flush_buf, steps=10, warmup=3):
+    """the naive state-dict copy -- one torch copy_ per tensor from
+    the producer's to the consumer's parameters (no snapshot, no seal, no
+    verification, no atomic swap: a reader can see a torn model).  Timed like
+    the update: CUDA events around the copies, L2 flushed before each."""
+    import torch
+    specs = synth.model_specs(name)
+    pt, ct = G.alloc_model(specs), G.alloc_model(specs)
+    st = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ms = []
+    for i in range(warmup + steps):
+        G.l2_flush(flush_buf, stream=st)
+        torch.cuda.synchronize()
+        e0.record(st)
+        for d, s in zip(ct, pt):
+            d.copy_(s)
+        e1.record(st)
+        e1.synchronize()
+        if i >= warmup:
+            ms.append(e0.elapsed_time(e1))
+    del pt, ct
+    return statistics.mean(ms)
+
+
 def event_floor_us(G, reps=20):
     """An empty kernel bracketed exactly like the library's timing events."""
     import torch
@@ -607,6 +632,14 @@ def gpu_arm(args):
                 out["c5_schedule"] = c5_schedule(V, G, synth, flush, sweep.get("llama3_8b", {}))
             except Exception as ex:
                 out["c5_schedule"] = {"error": str(ex)[:200]}
+        try:
+            base = {name: round(torch_copy_baseline(G, synth, name, flush), 6)}
+            if not args.no_sweep:
+                for nm in ["resnet50", "vit_b16", "gpt2_xl"]:
+                    base[nm] = round(torch_copy_baseline(G, synth, nm, flush), 6)
+            out["baseline_torch_state_dict_copy_ms"] = base
+        except Exception as ex:
+            out["baseline_torch_state_dict_copy_ms"] = {"error": str(ex)[:200]}
         out["cpu_baseline"] = cpu_baseline(synth, name, budget_s=args.cpu_budget)
         print(json.dumps(out), flush=True)
     if world > 1:
