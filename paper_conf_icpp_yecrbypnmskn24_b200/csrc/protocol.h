@@ -8,7 +8,9 @@
 //   reader               s <- state; ref[slot]++; re-read state  (try_acquire_slot)
 // All seq_cst std::atomic on words that may live in a shared-memory segment.
 #pragma once
+#include <errno.h>
 #include <sched.h>
+#include <signal.h>
 
 #include <atomic>
 #include <cstdint>
@@ -17,17 +19,31 @@
 
 namespace vp {
 
+// Failure detection: a consumer whose process no longer exists is marked
+// inactive (its pin and refcounts no longer hold anything back).
+inline bool consumer_alive(ConsRec *r) {
+    const int32_t pid = r->pid.load();
+    if (pid <= 0) return true;  // in-process consumer
+    if (kill(pid, 0) == -1 && errno == ESRCH) {
+        r->active.store(0);
+        return false;
+    }
+    return true;
+}
+
 // Producer: before overwriting the snapshot slot that holds old_v, wait until
 // no active consumer pins old_v.  Returns false (and *who) on timeout.
 inline bool wait_unpinned(Ctrl *ctrl, uint64_t old_v, int64_t timeout_ns, int *who) {
     const int nc = ctrl->ncons.load();
     for (int i = 0; i < nc; i++) {
         const int64_t w0 = now_ns();
+        uint32_t spins = 0;
         while (ctrl->cons[i].active.load() && ctrl->cons[i].pin.load() == old_v) {
             if (now_ns() - w0 > timeout_ns) {
                 if (who) *who = i;
                 return false;
             }
+            if ((++spins & 0xFFFF) == 0 && !consumer_alive(&ctrl->cons[i])) break;
             __builtin_ia32_pause();
         }
     }

@@ -40,6 +40,7 @@ struct alignas(64) ConsRec {
     std::atomic<uint32_t> done_seq;      // futex word, bumped after each install attempt
     std::atomic<int32_t> waiters;        // threads sleeping on done_seq
     std::atomic<int32_t> last_status;
+    std::atomic<int32_t> pid;            // consumer process (failure detection), 0 = in-process
     std::atomic<uint64_t> p1_done;       // scatter-allgather: phase-1 version finished
     std::atomic<uint64_t> p2_done;       // scatter-allgather: phase-2 version finished
 };

@@ -26,6 +26,7 @@
 #include <new>
 #include <random>
 
+#include "protocol.h"
 #include "runtime.h"
 
 namespace vp {
@@ -337,7 +338,10 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         }
         if (st == VIPER_OK && sa) st = open_sa_peers(m, all, bs);
         if (st == VIPER_OK && M > 1) st = open_producers(m, all, bs);
-        if (st == VIPER_OK) m->rec->active.store(1);
+        if (st == VIPER_OK) {
+            m->rec->pid.store((int32_t)getpid());
+            m->rec->active.store(1);
+        }
     }
     // ---- allgather #2: statuses (all ranks fail together)
     PeerRec fin{};
@@ -415,6 +419,10 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
         for (;;) {
             const uint32_t seq = r->done_seq.load();
             if (!r->active.load() || r->done_version.load() >= v) break;
+            if (!consumer_alive(r)) {  // its process exited: stop waiting, report it
+                if (worst == VIPER_OK) worst = set_error(VIPER_E_PEER, "consumer %d exited", i);
+                break;
+            }
             if (now_ns() - t0 > 60ll * 1000000000ll)
                 return set_error(VIPER_E_TIMEOUT, "consumer %d did not install v%llu", i, (unsigned long long)v);
             r->waiters.fetch_add(1);

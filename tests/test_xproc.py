@@ -89,6 +89,16 @@ def test_xproc_data_parallel_producers(nproc, nprod, mode, config):
 
 
 @pytest.mark.gpu
+def test_xproc_consumer_process_death_is_detected():
+    """A consumer process exits without unregistering: the SYNC producer notices
+    (pid liveness in the shared control block) instead of stalling, and the
+    surviving consumer keeps installing every version."""
+    rc, out = run_torchrun(3, "tests/xproc_fail_worker.py", [], timeout=180)
+    assert "FAIL_PRODUCER" in out and "ok=True" in out, out[-4000:]
+    assert "FAIL_SURVIVOR version=6 good=True" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 def test_xproc_fault_injection():
     rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fault", "1", "--versions", "3"])
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
