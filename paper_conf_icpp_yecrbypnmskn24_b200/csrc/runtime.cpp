@@ -551,7 +551,8 @@ viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
 }
 
 int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug_trace)
-#define TRACE(i) (g_trace[i] = now_ns())
+static const bool g_trace_on = getenv("VIPER_TRACE") != nullptr;  // tools/trace_publish.py sets it
+#define TRACE(i) (g_trace_on ? (void)(g_trace[i] = now_ns()) : (void)0)
 
 // The fused kernel through a one-node CUDA graph whose parameters are updated
 // per publish: measured cheaper on the host than a direct launch
@@ -584,7 +585,7 @@ std::atomic<uint64_t> &pub_word(viper_model *p) {
 static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st) {
     NvtxRange nvtx("viper_publish");
     const int64_t t0 = now_ns();
-    g_trace[0] = t0;
+    if (g_trace_on) g_trace[0] = t0;
     if (v == 0 || v <= p->last_version)
         return set_error(VIPER_E_VERSION, "publish(%llu) after %llu: versions strictly increase from 1",
                          (unsigned long long)v, (unsigned long long)p->last_version);

@@ -1,6 +1,8 @@
 """Host-side breakdown of one SYNC publish (debug trace timestamps)."""
 import ctypes as C
 import os
+
+os.environ.setdefault("VIPER_TRACE", "1")
 import statistics
 import sys
 import time
