@@ -425,6 +425,10 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
             }
             if (now_ns() - t0 > 60ll * 1000000000ll)
                 return set_error(VIPER_E_TIMEOUT, "consumer %d did not install v%llu", i, (unsigned long long)v);
+            if (now_ns() - t0 < 200000) {  // spin first: a futex wake-up costs tens of us
+                __builtin_ia32_pause();
+                continue;
+            }
             r->waiters.fetch_add(1);
             if (r->done_seq.load() == seq && r->done_version.load() < v) futex_wait(&r->done_seq, seq, 1000);
             r->waiters.fetch_sub(1);
