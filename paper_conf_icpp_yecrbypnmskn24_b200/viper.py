@@ -190,8 +190,9 @@ class View:
 class _CAI:
     def __init__(self, ptr, t):
         import torch
-        typestr = {torch.float32: "<f4", torch.float16: "<f2", torch.uint8: "|u1", torch.int16: "<i2",
-                   torch.int32: "<i4"}[t.dtype if t.dtype != torch.bfloat16 else torch.int16]
+        typestr = {torch.float32: "<f4", torch.float16: "<f2", torch.float64: "<f8", torch.uint8: "|u1",
+                   torch.int8: "|i1", torch.int16: "<i2", torch.int32: "<i4", torch.int64: "<i8",
+                   torch.bool: "|b1"}[t.dtype if t.dtype != torch.bfloat16 else torch.int16]
         self.__cuda_array_interface__ = {"shape": tuple(t.shape), "typestr": typestr, "data": (ptr, False),
                                          "version": 3, "strides": None}
 

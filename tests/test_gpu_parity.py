@@ -506,3 +506,16 @@ def test_randomized_configurations(seed):
         assert np.array_equal(p_dev, p_or) and np.array_equal(s_dev, s_or)
     finally:
         close_all(prod, cons)
+
+
+def test_example_train_and_serve():
+    """examples/train_and_serve.py: real ResNet-18 training publishes ASYNC while
+    an inference thread serves; the served logits equal the trainer's."""
+    import importlib.util
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    spec = importlib.util.spec_from_file_location("tas", os.path.join(root, "examples", "train_and_serve.py"))
+    tas = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(tas)
+    same, served = tas.main(steps=30, every=3, verbose=False)
+    assert same
+    assert served["n"] > 0 and len(served["versions"]) >= 2
