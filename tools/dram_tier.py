@@ -42,3 +42,27 @@ for name, fn in (("D2H", lambda: h.copy_(d, non_blocking=True)), ("H2D", lambda:
     t0 = time.perf_counter(); fn(); torch.cuda.synchronize()
     dt = time.perf_counter() - t0
     print(f"pinned {name} {S/1e9:.2f} GB: {S / dt / 1e9:.1f} GB/s", flush=True)
+
+# bidirectional: a D2H and an H2D of the same size at once on two streams
+# (the DRAM tier's steady state: the producer's D2H of piece i overlaps the
+# consumer's H2D of piece i-1)
+nb = min(S, 4 << 30)
+ha, hb = G.PinnedBuffer(nb), G.PinnedBuffer(nb)
+da = torch.empty(nb, dtype=torch.uint8, device="cuda")
+db = torch.empty(nb, dtype=torch.uint8, device="cuda")
+sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+for rep in range(2):
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ha.from_device_ptr(da.data_ptr(), nb, stream=sa)
+    hb.to_device(db, stream=sb)
+    torch.cuda.synchronize()
+    dt = time.perf_counter() - t0
+print(f"pinned D2H || H2D {nb/1e9:.2f} GB each: {nb / dt / 1e9:.1f} GB/s per direction, {2 * nb / dt / 1e9:.1f} GB/s total",
+      flush=True)
+for name, fn in (("D2H", lambda: ha.from_device_ptr(da.data_ptr(), nb, stream=sa)), ("H2D", lambda: hb.to_device(db, stream=sa))):
+    fn(); torch.cuda.synchronize()
+    t0 = time.perf_counter(); fn(); torch.cuda.synchronize()
+    dt = time.perf_counter() - t0
+    print(f"raw pinned {name} {nb/1e9:.2f} GB alone: {nb / dt / 1e9:.1f} GB/s", flush=True)
+ha.close(); hb.close()
