@@ -281,8 +281,7 @@ extern "C" viper_status viper_restore(const char *path, const viper_tensor *tens
             a.iseal = (const ISeal *)d;
             a.version = hd.version;
             a.fault_item = ~0u;
-            a.done = (uint32_t *)flags;
-            a.err = (uint32_t *)flags + 1;
+            a.flags = (unsigned long long *)flags;
             a.status_h = (volatile int32_t *)sh_dev;
             e = launch_install(a, pick_geometry(a.nitems, device), s, false);
         }

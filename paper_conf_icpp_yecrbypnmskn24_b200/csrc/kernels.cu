@@ -278,25 +278,41 @@ __global__ void seal_reduce_kernel(const SealReduceArgs a) {
     }
 }
 
+// Grid completion word: low 32 bits count finished blocks, high 32 bits carry
+// error bits.  Both halves live in ONE 64-bit word updated only by 64-bit
+// atomics, so the last block's arrival returns every error reported before
+// it.  This saves the separate error exchange (one L2 round trip) on the
+// critical path.
+__device__ __forceinline__ void report_err(unsigned long long *flags, uint32_t bits) {
+    atomicOr(flags, (unsigned long long)bits << 32);
+}
+
+// Thread 0 of each block, after __syncthreads: release this block's stores
+// (bar.sync + a gpu-scope release is cumulative over the block) and count it.
+// Returns true in the last block, with the grid's error bits, and resets the word.
+__device__ __forceinline__ bool grid_arrive(unsigned long long *flags, uint32_t *err) {
+    unsigned long long old;
+    asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], 1;" : "=l"(old) : "l"(flags) : "memory");
+    if ((uint32_t)old != gridDim.x - 1) return false;
+    *err = (uint32_t)(old >> 32);
+    *flags = 0;  // every block has arrived: nobody else touches it in this grid
+    return true;
+}
+
 // End of an install grid: the last block to finish publishes the result and,
 // when every item matched, swaps the version word from the device.
 __device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
-    if (bad) atomicOr(a.err, kErrChecksum);
+    if (bad) report_err(a.flags, kErrChecksum);
     __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();  // cumulative over the block's stores (ordered by the barrier)
-        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
-            __threadfence();
-            const uint32_t e = atomicExch(a.err, 0u);
-            *a.done = 0;
-            const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
-            // Every block's slot stores are GPU-visible (cumulative fences
-            // above); later readers are kernels launched after the host saw
-            // the flip, so plain system-visible stores suffice here.
-            if (a.status_h) *a.status_h = st;
-            if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
-            if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
-        }
+    uint32_t e;
+    if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
+        const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
+        // Every block's slot stores are GPU-visible (released by its arrival,
+        // acquired by this one); later readers are kernels launched after the
+        // host saw the flip, so plain system-visible stores suffice here.
+        if (a.status_h) *a.status_h = st;
+        if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
+        if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
     }
 }
 
@@ -360,7 +376,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                 waited += backoff;
                 if (backoff < 1024) backoff <<= 1;
                 if (waited > kItemWaitNs) {  // never hang on a vanished producer
-                    atomicOr(a.err, kErrTimeout);
+                    report_err(a.flags, kErrTimeout);
                     break;
                 }
             }
@@ -444,21 +460,16 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
             if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
         }
     }
-    if (lane == 0 && bad) atomicOr(a.err, bad);
+    if (lane == 0 && bad) report_err(a.flags, bad);
     __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        if (atomicAdd(a.done, 1u) == gridDim.x - 1) {
-            __threadfence();
-            const uint32_t e = atomicExch(a.err, 0u);
-            *a.done = 0;
-            for (uint32_t k = 0; k < a.ncons; k++) {
-                const FusedCons &c = a.cons[k];
-                const int32_t st = (e >> k) & 1u ? -5 : 0;
-                if (c.status_h) *c.status_h = st;
-                if (st == 0 && c.state_h) *c.state_h = (a.version << 1) | (uint64_t)c.target;  // the swap
-                if (c.pin_h) *c.pin_h = 0;
-            }
+    uint32_t e;
+    if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
+        for (uint32_t k = 0; k < a.ncons; k++) {
+            const FusedCons &c = a.cons[k];
+            const int32_t st = (e >> k) & 1u ? -5 : 0;
+            if (c.status_h) *c.status_h = st;
+            if (st == 0 && c.state_h) *c.state_h = (a.version << 1) | (uint64_t)c.target;  // the swap
+            if (c.pin_h) *c.pin_h = 0;
         }
     }
 }
@@ -669,7 +680,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
             while (ld_acquire_sys(&is->version) != a.version) {
                 __nanosleep(256);
                 if ((waited += 256) > kItemWaitNs) {
-                    atomicOr(a.err, kErrTimeout);
+                    report_err(a.flags, kErrTimeout);
                     break;
                 }
             }
@@ -713,7 +724,8 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
         const uint64_t part = warp_sum(acc);
         if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
     }
-    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // slot stores complete
+    if (lane == 0)  // slot stores complete, then ordered before the generic-proxy release below
+        asm volatile("cp.async.bulk.wait_group 0;\n\tfence.proxy.async.global;" ::: "memory");
     __syncwarp();
     install_finish(a, bad);
 }

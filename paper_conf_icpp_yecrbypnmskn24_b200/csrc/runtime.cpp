@@ -343,8 +343,7 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
     a.target = (uint32_t)target;
     a.fault_item = ~0u;
     if (c->fault_next.exchange(false) && a.nitems) a.fault_item = a.nitems / 2;
-    a.done = c->d_flags;
-    a.err = c->d_flags + 1;
+    a.flags = (unsigned long long *)c->d_flags;
     a.status_h = (volatile int32_t *)&c->rec_dev->status;
     a.pin_h = (volatile uint64_t *)&c->rec_dev->pin;
     a.state_h = (volatile uint64_t *)&c->rec_dev->state;
@@ -662,8 +661,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         f.packed = p->d_snap[b];
         f.iseal = p->d_iseal[b];
         f.version = v;
-        f.done = p->d_flags;
-        f.err = p->d_flags + 1;
+        f.flags = (unsigned long long *)p->d_flags;
         for (size_t k = 0; k < prepared.size(); k++) {
             const InstallArgs &ia = prepared[k].a;
             f.cons[k] = FusedCons{ia.items, ia.target, ia.fault_item, ia.status_h, ia.pin_h, ia.state_h};

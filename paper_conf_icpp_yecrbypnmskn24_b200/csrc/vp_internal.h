@@ -70,8 +70,7 @@ struct InstallArgs {
     uint64_t version;
     uint32_t target;            // slot being written
     uint32_t fault_item;        // item whose first word is flipped (fault injection); ~0u = none
-    uint32_t *done;             // [1] blocks finished (self-resetting)
-    uint32_t *err;              // [1] error bits (self-resetting)
+    unsigned long long *flags;  // [1] low 32 bits: blocks finished; high 32: error bits (self-resetting)
     // Host-mapped control words (cudaHostAlloc/cudaHostRegister mapped).  The
     // last block writes *status_h, clears *pin_h and, when every item matched,
     // flips *state_h = (version << 1) | target: the atomic version swap.
@@ -116,8 +115,7 @@ struct FusedArgs {
     uint8_t *packed;
     ISeal *iseal;
     uint64_t version;
-    uint32_t *done;             // [1] self-resetting
-    uint32_t *err;              // [1] bit k = consumer k failed, self-resetting
+    unsigned long long *flags;  // [1] low 32: blocks finished; high 32: bit k = consumer k failed (self-resetting)
     FusedCons cons[kMaxFused];
 };
 
