@@ -643,6 +643,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         }
     }
     TRACE(2);
+    if (p->xproc && p->early_notify) {  // v is named when the stream reaches the pack (xproc.cpp)
+        viper_status s = xproc_notify_early(p, v, b, st);
+        if (s) return s;
+    }
     const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
     std::vector<viper_model *> launched;
     // TMA bulk-copy pack: forced by the flag, or auto for packs no install is
@@ -714,16 +718,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     p->snap_version[b] = v;
     p->cur_snap = b;
     p->last_version = v;
-    if (!p->xproc || p->early_notify) {
-        // in process, consumers order themselves after ev_ready[b]; across
-        // GPUs with early notification their install waits per item on the
-        // seals the pack releases at system scope (cross-GPU pipeline)
+    if (!p->xproc) {
+        // in process, consumers order themselves after ev_ready[b]
         pub_word(p).store((v << 1) | (uint64_t)b);
         ctrl->pub_time_ns.store(now_ns());
-        if (p->xproc) {
-            ctrl->pub_seq.fetch_add(1);
-            futex_wake_all(&ctrl->pub_seq);
-        }
     }
     // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
@@ -863,6 +861,7 @@ static void free_model(viper_model *m) {
         for (int k = 0; k < 2; k++)
             if (evs[k]) cudaEventDestroy(evs[k]);
     if (m->ev_packed) cudaEventDestroy(m->ev_packed);
+    if (m->ev_notify) cudaEventDestroy(m->ev_notify);
     if (m->fused_exec) cudaGraphExecDestroy(m->fused_exec);
     if (m->fused_graph) cudaGraphDestroy(m->fused_graph);
     if (m->side) cudaStreamDestroy(m->side);
@@ -895,6 +894,7 @@ viper_status alloc_producer(viper_model *m, const viper_tensor *tensors) {
     for (auto &e : m->ev_sealed) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     for (auto &e : m->ev_t) CUDA_TRY(cudaEventCreate(&e));
     CUDA_TRY(cudaEventCreateWithFlags(&m->ev_packed, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreateWithFlags(&m->ev_notify, cudaEventDisableTiming));
     CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
     CUDA_TRY(cudaMalloc(&m->d_flags, 64));
     CUDA_TRY(cudaMemset(m->d_flags, 0, 64));

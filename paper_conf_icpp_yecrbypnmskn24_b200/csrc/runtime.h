@@ -129,6 +129,7 @@ struct viper_model {
     void *snap_alloc = nullptr;
     cudaEvent_t ev_ready[2] = {nullptr, nullptr};   // snapshot slot b complete
     cudaEvent_t ev_packed = nullptr;
+    cudaEvent_t ev_notify = nullptr;   // producer, early notification: the stream reached the pack
     cudaEvent_t ev_t[2] = {nullptr, nullptr};        // VIPER_FLAG_TIMING: around the kernel
     bool timing_pending = false;
     bool last_fused = false;                         // last publish used publish_fused_kernel
@@ -251,6 +252,7 @@ void flush_stats(viper_model *m, uint64_t *flushed, uint64_t *skipped, uint64_t 
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs);
 viper_status xproc_install(viper_model *c, uint64_t v, int b);   // consumer update thread
 viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool already = false);  // producer
+viper_status xproc_notify_early(viper_model *p, uint64_t v, int b, cudaStream_t st);           // producer
 void xproc_free(viper_model *m);
 
 }  // namespace vp

@@ -142,6 +142,18 @@ void CUDART_CB notify_fn(void *p) {  // host function: no CUDA calls here
     delete n;
 }
 
+struct WakeCtx {
+    Ctrl *ctrl;
+};
+
+void CUDART_CB wake_fn(void *p) {  // host function: wake sleeping consumers (the word is already set)
+    WakeCtx *w = (WakeCtx *)p;
+    w->ctrl->pub_time_ns.store(now_ns());
+    w->ctrl->pub_seq.fetch_add(1);
+    futex_wake_all(&w->ctrl->pub_seq);
+    delete w;
+}
+
 viper_status open_sa_peers(viper_model *m, const std::vector<PeerRec> &all, const viper_bootstrap *bs) {
     const int N = m->nconsumers_x;
     std::vector<const uint8_t *> src(2 * N), isrc(2 * N);
@@ -437,6 +449,29 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
             worst = set_error(r->last_status.load(), "consumer %d failed to install v%llu", i, (unsigned long long)v);
     }
     return worst;
+}
+
+// Early notification (every consumer on another GPU): consumers launch install
+// grids that wait per item on the seals the pack releases at system scope, so
+// pack, NVLink pull and install overlap.  v is named by a stream memop placed
+// right BEFORE the pack: a consumer GPU starts spinning on item seals only
+// once the training stream has drained its earlier work and reached the pack,
+// not at host enqueue time.  Sleeping update threads are then woken by a host
+// function on the side stream (it does not write the word, so a late wake-up
+// never names an older version over a newer one).
+viper_status xproc_notify_early(viper_model *p, uint64_t v, int b, cudaStream_t st) {
+    void *dev_word = p->nprod > 1 ? (void *)&p->ctrl_dev->pub_m[p->pidx] : (void *)&p->ctrl_dev->pub_state;
+    viper_status s = stream_write(st, dev_word, (v << 1) | (uint64_t)b);
+    if (s) return s;
+    CUDA_TRY(cudaEventRecord(p->ev_notify, st));
+    CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_notify, 0));
+    WakeCtx *w = new WakeCtx{p->ctrl};
+    const cudaError_t e = cudaLaunchHostFunc(p->side, wake_fn, w);
+    if (e != cudaSuccess) {
+        delete w;
+        return set_error(VIPER_E_CUDA, "cudaLaunchHostFunc: %s", cudaGetErrorString(e));
+    }
+    return VIPER_OK;
 }
 
 void xproc_free(viper_model *m) {

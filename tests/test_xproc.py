@@ -70,6 +70,17 @@ def test_xproc_early_notify_pipeline(nproc, fanout, mode):
 
 
 @pytest.mark.gpu
+def test_xproc_early_notify_waits_for_the_stream():
+    """Early notification names v by a stream memop right before the pack: with
+    300 ms of earlier work queued on the producer's stream, a consumer's install
+    (launch -> done) stays short instead of spinning on its GPU for 300 ms."""
+    rc, out = run_torchrun(2, "tests/xproc_worker.py",
+                           ["--config", "resnet50", "--mode", "1", "--versions", "3", "--delay-ms", "300"],
+                           env={"VIPER_EARLY_NOTIFY": "1"})
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 @pytest.mark.parametrize("nproc,fanout", [(3, 0), (4, 2)])
 def test_xproc_no_torn_reads(nproc, fanout):
     rc, out = run_torchrun(nproc, "tests/xproc_worker.py", ["--config", "small", "--mode", "1", "--fanout",

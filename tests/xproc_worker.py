@@ -79,6 +79,9 @@ def main():
     ap.add_argument("--fault", type=int, default=0)
     ap.add_argument("--stress", type=int, default=0, help="ASYNC publishes while consumers verify every view")
     ap.add_argument("--nprod", type=int, default=1, help="data-parallel producers (ranks 0..nprod-1)")
+    ap.add_argument("--delay-ms", type=float, default=0.0,
+                    help="ASYNC: the producer's stream sleeps this long before each publish; consumers check "
+                         "that their install did not start (and spin) before the stream reached the pack")
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
@@ -105,6 +108,8 @@ def main():
         if is_prod:
             G.fill_model(tensors, specs, seed, v)
             torch.cuda.synchronize()
+            if a.delay_ms:
+                torch.cuda._sleep(int(a.delay_ms * 2.0e6))  # ~2 GHz SM clock
             try:
                 m.publish(v)
             except V.ViperError as e:
@@ -151,7 +156,11 @@ def main():
                 errors += 1
         m.release(view)
         st = m.stats()
-        print(f"[rank{rank}] installs={st['installs']} skipped={st['skipped']}", flush=True)
+        print(f"[rank{rank}] installs={st['installs']} skipped={st['skipped']} "
+              f"last install {st['t_install_us']:.0f} us", flush=True)
+        if a.delay_ms and st["t_install_us"] > a.delay_ms * 1e3 / 3:
+            print(f"[rank{rank}] install started before the producer's stream reached the pack", flush=True)
+            errors += 1
     dist.barrier()
     if not is_prod:
         m.close()
