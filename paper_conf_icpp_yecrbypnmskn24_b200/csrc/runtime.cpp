@@ -978,9 +978,29 @@ using namespace vp;
 extern "C" {
 
 
-viper_status viper_register_model(const char *model_name, int32_t role, const viper_tensor *tensors, int32_t n,
-                                  const viper_config *cfg, const viper_bootstrap *bs, viper_model **out) {
-    try {
+// Every tensor must be device (or managed) memory of the model's device: a
+// tensor on another GPU would otherwise be read over the peer mapping, or fault.
+static viper_status check_tensor_devices(const viper_tensor *t, int32_t n, int device) {
+    for (int32_t i = 0; i < n; i++) {
+        if (!t[i].nbytes) continue;
+        cudaPointerAttributes pa{};
+        if (cudaPointerGetAttributes(&pa, t[i].dev_ptr) != cudaSuccess) {
+            cudaGetLastError();
+            return set_error(VIPER_E_INVAL, "tensor %d: not a CUDA allocation", i);
+        }
+        if (pa.type == cudaMemoryTypeManaged) continue;
+        if (pa.type != cudaMemoryTypeDevice)
+            return set_error(VIPER_E_INVAL, "tensor %d: not device memory (there is no host path)", i);
+        if (pa.device != device)
+            return set_error(VIPER_E_INVAL, "tensor %d lives on device %d, the model on device %d", i, pa.device, device);
+    }
+    return VIPER_OK;
+}
+
+static viper_status register_impl(const char *model_name, int32_t role, const viper_tensor *tensors, int32_t n,
+                                  const viper_config *cfg, const viper_bootstrap *bs, viper_model **out,
+                                  bool *joined) {
+    {
         if (!out) return set_error(VIPER_E_INVAL, "out is NULL");
         *out = nullptr;
         if (!model_name || !*model_name) return set_error(VIPER_E_INVAL, "empty model name");
@@ -1002,6 +1022,8 @@ viper_status viper_register_model(const char *model_name, int32_t role, const vi
             return set_error(VIPER_E_CUDA, "no CUDA device (there is no CPU fallback)");
         if (c.device < 0 || c.device >= ndev) return set_error(VIPER_E_INVAL, "bad device %d", c.device);
         CUDA_TRY(cudaSetDevice(c.device));
+        st = check_tensor_devices(tensors, n, c.device);
+        if (st) return st;
         viper_model *m = new viper_model();
         m->name = model_name;
         m->role = role;
@@ -1012,6 +1034,7 @@ viper_status viper_register_model(const char *model_name, int32_t role, const vi
             m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device);
             if (bs && bs->world > 1) {
                 m->xproc = true;
+                *joined = true;
                 st = xproc_register(m, tensors, bs);
             } else {
                 st = register_local(m, tensors);
@@ -1031,9 +1054,22 @@ viper_status viper_register_model(const char *model_name, int32_t role, const vi
         }
         *out = m;
         return VIPER_OK;
-    } catch (const std::exception &e) {
-        return set_error(VIPER_E_NOMEM, "register: %s", e.what());
     }
+}
+
+viper_status viper_register_model(const char *model_name, int32_t role, const viper_tensor *tensors, int32_t n,
+                                  const viper_config *cfg, const viper_bootstrap *bs, viper_model **out) {
+    bool joined = false;
+    viper_status st;
+    try {
+        st = register_impl(model_name, role, tensors, n, cfg, bs, out, &joined);
+    } catch (const std::exception &e) {
+        st = set_error(VIPER_E_NOMEM, "register: %s", e.what());
+    }
+    // failed before the bootstrap: still take part in its collectives, so the
+    // other ranks fail with VIPER_E_PEER instead of waiting forever
+    if (st != VIPER_OK && !joined && bs && bs->world > 1 && bs->allgather) xproc_abort(bs, st);
+    return st;
 }
 
 viper_status viper_publish(viper_model *m, uint64_t version, void *cuda_stream) {

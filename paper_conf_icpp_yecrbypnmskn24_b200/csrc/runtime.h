@@ -253,6 +253,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
 viper_status xproc_install(viper_model *c, uint64_t v, int b);   // consumer update thread
 viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool already = false);  // producer
 viper_status xproc_notify_early(viper_model *p, uint64_t v, int b, cudaStream_t st);           // producer
+void xproc_abort(const viper_bootstrap *bs, viper_status st);  // failed before the bootstrap
 void xproc_free(viper_model *m);
 
 }  // namespace vp

@@ -213,12 +213,18 @@ viper_status open_producers(viper_model *m, const std::vector<PeerRec> &all, con
 
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs) {
     if (!bs->allgather) return set_error(VIPER_E_INVAL, "bootstrap.allgather is NULL");
-    if (bs->rank < 0 || bs->rank >= bs->world || bs->producer_rank < 0 || bs->producer_rank >= bs->world)
-        return set_error(VIPER_E_INVAL, "bad bootstrap ranks");
     const int M = bs->nproducers > 1 ? bs->nproducers : 1;
-    if (M > kMaxProducers || bs->producer_rank + M > bs->world)
-        return set_error(VIPER_E_INVAL, "bad nproducers %d", bs->nproducers);
-    if (bs->world - M > kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+    viper_status bad = VIPER_OK;
+    if (bs->rank < 0 || bs->rank >= bs->world || bs->producer_rank < 0 || bs->producer_rank >= bs->world)
+        bad = set_error(VIPER_E_INVAL, "bad bootstrap ranks");
+    else if (M > kMaxProducers || bs->producer_rank + M > bs->world)
+        bad = set_error(VIPER_E_INVAL, "bad nproducers %d", bs->nproducers);
+    else if (bs->world - M > kMaxConsumers)
+        bad = set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+    if (bad) {  // still take part in the bootstrap collectives: the peers fail instead of hanging
+        xproc_abort(bs, bad);  // (does not touch the error text)
+        return bad;
+    }
     m->rank = bs->rank;
     m->world = bs->world;
     m->nconsumers_x = bs->world - M;
@@ -367,6 +373,16 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         if (sts[r].status != VIPER_OK) return set_error(VIPER_E_PEER, "rank %d failed to register", r);
     if (!producer) m->upd = std::thread(update_loop, m);
     return VIPER_OK;
+}
+
+void xproc_abort(const viper_bootstrap *bs, viper_status st) {
+    PeerRec me{};
+    me.magic = kPeerMagic;
+    me.rank = bs->rank;
+    me.status = st;
+    std::vector<PeerRec> all(bs->world > 0 ? bs->world : 1);
+    if (bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user) != 0) return;
+    bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user);
 }
 
 // Consumer update thread (install_mu held, v pinned): pull slot b of the

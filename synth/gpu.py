@@ -46,9 +46,11 @@ def fill_model(tensors, specs, seed: int, version: int, stream=None):
         fill(t, seed, version, i, s[1], stream)
 
 
-def alloc_model(specs, device="cuda:0"):
-    """Allocate one CUDA tensor per spec (torch dtype matching the spec)."""
+def alloc_model(specs, device=None):
+    """Allocate one CUDA tensor per spec (torch dtype matching the spec), on
+    `device` or else on the current CUDA device (one process per GPU)."""
     import torch
+    device = device if device is not None else torch.device("cuda", torch.cuda.current_device())
     from . import F32, BF16, F16
     dt = {F32: torch.float32, BF16: torch.bfloat16, F16: torch.float16}
     return [torch.empty(s[2], dtype=dt.get(s[1], torch.uint8), device=device) for s in specs]

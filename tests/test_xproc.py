@@ -120,6 +120,21 @@ def test_bootstrap_allgather_gloo_world2():
     assert rc == 0 and "BOOTSTRAP_OK" in out, out[-3000:]
 
 
+def test_bootstrap_pre_failure_does_not_hang():
+    """A rank failing before the bootstrap still joins its allgathers (CPU: both
+    ranks fail with "no CUDA device"; GPU box: rank 1's host tensor is rejected
+    and rank 0 gets VIPER_E_PEER)."""
+    rc, out = run_torchrun(2, "tests/bootstrap_abort_worker.py", [], timeout=120)
+    assert rc == 0 and "ABORT_OK" in out, out[-3000:]
+
+
+@pytest.mark.gpu
+def test_bootstrap_pre_failure_does_not_hang_gpu():
+    """Same on a GPU box: rank 0 reaches the bootstrap and must fail with VIPER_E_PEER."""
+    rc, out = run_torchrun(2, "tests/bootstrap_abort_worker.py", [], timeout=120)
+    assert rc == 0 and "ABORT_OK" in out, out[-3000:]
+
+
 def test_protocol_two_processes_gloo_cpu():
     """The cross-process version protocol on a real shm segment, CPU only:
     0 torn snapshot copies, 0 torn reads, no version regress over 3000 publishes."""
