@@ -179,9 +179,12 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
         m.chunk_first[c + 1] = m.chunk_first[c] + per_chunk[c];
     }
     if (m.items.size() >= (size_t)UINT32_MAX) return set_error(VIPER_E_INVAL, "too many work items");
-    // DRAM-tier pipeline pieces: whole chunks, >= 32 MiB, at most kMaxPieces
+    // DRAM-tier pipeline pieces: whole chunks, about S/64 clamped to
+    // [8 MiB, 64 MiB] (VIPER_DRAM_PIECE overrides, for sweeps), at most kMaxPieces
     {
-        const uint64_t want = std::max<uint64_t>(32ull << 20, (m.s_packed + kMaxPieces - 1) / kMaxPieces);
+        uint64_t want = std::min<uint64_t>(std::max<uint64_t>(m.s_packed / 64, 8ull << 20), 64ull << 20);
+        if (const char *e = getenv("VIPER_DRAM_PIECE")) want = std::max<uint64_t>(strtoull(e, nullptr, 10), 1);
+        want = std::max<uint64_t>(want, (m.s_packed + kMaxPieces - 1) / kMaxPieces);
         const uint64_t per = std::max<uint64_t>(1, (want + chunk_bytes - 1) / chunk_bytes);  // chunks per piece
         m.piece_lo.clear(); m.piece_hi.clear(); m.piece_ilo.clear(); m.piece_ihi.clear();
         for (uint64_t c = 0; c < m.nchunks; c += per) {

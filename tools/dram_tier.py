@@ -15,11 +15,12 @@ from synth import gpu as G
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="resnet50")
 ap.add_argument("--steps", type=int, default=4)
+ap.add_argument("--dram-only", action="store_true", help="only the DRAM-tier update (piece sweeps)")
 a = ap.parse_args()
 specs = synth.model_specs(a.config)
 S = synth.model_bytes(a.config)
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
-for tier in (V.TIER_DRAM, V.TIER_GPU):
+for tier in ((V.TIER_DRAM,) if a.dram_only else (V.TIER_DRAM, V.TIER_GPU)):
     c = V.Model(f"d{tier}", V.CONSUMER, ct, tier=tier)
     p = V.Model(f"d{tier}", V.PRODUCER, pt, tier=tier)
     lat = []
@@ -34,6 +35,8 @@ for tier in (V.TIER_DRAM, V.TIER_GPU):
           f"({S / (statistics.mean(lat) * 1e-3) / 1e9:.1f} GB/s)", flush=True)
     c.close()
     p.close()
+if a.dram_only:
+    sys.exit(0)
 # raw pinned copy rates
 h = torch.empty(S, dtype=torch.uint8).pin_memory()
 d = torch.empty(S, dtype=torch.uint8, device="cuda")
