@@ -350,16 +350,18 @@ def test_no_torn_reads_under_async_publishes():
 
 
 # ----------------------------------------------- BJ-sized models in 1-GPU loopback
-@pytest.mark.parametrize("name,flags", [("resnet50", 0), ("vit_b16", 0), ("gpt2_xl", 0), ("llama3_8b", 0),
-                                        ("gpt2_xl", V.FLAG_TMA)])
-def test_full_size_loopback_sampled(name, flags):
+@pytest.mark.parametrize("name,flags,tier", [("resnet50", 0, V.TIER_GPU), ("vit_b16", 0, V.TIER_GPU),
+                                             ("gpt2_xl", 0, V.TIER_GPU), ("llama3_8b", 0, V.TIER_GPU),
+                                             ("gpt2_xl", V.FLAG_TMA, V.TIER_GPU), ("resnet50", 0, V.TIER_DRAM),
+                                             ("gpt2_xl", 0, V.TIER_DRAM)])
+def test_full_size_loopback_sampled(name, flags, tier):
     """Full BASELINE.json model sizes, single-GPU loopback (the launch config
     bench.py times): every seal's version; sampled chunk seals recomputed by the
     oracle; sampled tensor byte ranges vs VGEN; all slot tensors == producer
     tensors (replica identity at any size)."""
     specs = synth.model_specs(name)
     seed = synth.SEEDS[name]
-    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.SYNC, flags=flags)
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, mode=V.SYNC, flags=flags, tier=tier)
     try:
         for v in (1, 2):
             G.fill_model(prod_t, specs, seed, v)
@@ -389,6 +391,32 @@ def test_full_size_loopback_sampled(name, flags):
     finally:
         close_all(prod, cons)
         torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("mode", [V.SYNC, V.ASYNC])
+def test_dram_tier_many_pieces(mode, monkeypatch):
+    """The DRAM tier's D2H -> H2D piece pipeline with the maximum piece count
+    (256 pieces of whole 4 KiB chunks): bytes and chunk seals equal the oracle's."""
+    monkeypatch.setenv("VIPER_DRAM_PIECE", "1")  # -> S/256 per piece, rounded to whole chunks
+    rng = np.random.default_rng(11)
+    specs = [(f"t{i}", synth.F32 if i % 3 else synth.BYTES, (int(rng.integers(1, 70_000)),)) for i in range(40)]
+    seed = 0x91EC
+    prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=2, mode=mode, tier=V.TIER_DRAM, chunk_bytes=4096)
+    try:
+        for v in range(1, 5):
+            G.fill_model(prod_t, specs, seed, v)
+            prod.publish(v)
+        for c, ct in zip(cons, cons_t):
+            c.wait_installed(4, timeout_us=20_000_000)
+            view = c.acquire_latest()
+            assert view.version == 4
+            check_slot(view, ct, specs, seed, 4)
+            c.release(view)
+        p_dev, s_dev = device_packed_and_seals(prod)
+        p_or, s_or, _ = oracle_packed_and_seals(specs, seed, 4, 4096)
+        assert np.array_equal(p_dev, p_or) and np.array_equal(s_dev, s_or)
+    finally:
+        close_all(prod, cons)
 
 
 def test_teardown_races_in_process():
