@@ -1,11 +1,14 @@
 #!/usr/bin/env python
 """bench.py -- model-update latency of the Viper hot path on B200.
 
-Default (N=1): BASELINE.json configs[0], the only single-GPU configuration:
-PtychoNN-sized fp32 model (40 tensors, 4.6 MB), 1 producer -> 1 consumer on
-one GPU (in-process loopback, GPU tier, SYNC mode).  One step = one versioned
-model update: pack + seal (K2) -> publish/notify -> install + verify (K6) ->
-device-side atomic version swap; publish() returns once the consumer serves v.
+Default (N=1): BASELINE.json configs[1], the first configuration the metric
+is quoted on, in 1-GPU form: ResNet-50 fp32 (161 tensors, 102 MB), 1 producer
+-> 1 consumer on one GPU (in-process loopback: the NVLink hop of configs[1]
+needs a second GPU; GPU tier, SYNC mode).  configs[0] (PtychoNN-sized, 4.6 MB)
+is the small parity case; it is reported in the loopback sweep beside the
+larger configs.  One step = one versioned model update: pack + seal (K2) ->
+publish/notify -> install + verify (K6) -> device-side atomic version swap;
+publish() returns once the consumer serves v.
 
 Timing: per step, L2 is flushed (a 256 MiB write, > the 126 MB L2) and the
 producer's tensors are rewritten with VGEN(v) (the synthetic "optimizer step")
@@ -56,6 +59,27 @@ def ncu_traffic(kernel, config):
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             t = json.load(f)
         return t.get(f"{kernel}:{config}", {}).get("traffic_bytes")
+    except Exception:
+        return None
+
+
+LAUNCH_LISTS = {"resnet50": "profiles/r01/launches_bench_r50_summary.json",
+                "ptychonn": "profiles/r01/launches_bench_c1_summary.json"}
+
+
+def ncu_launches(config, kernel, alg_bytes, peak):
+    """The committed ncu launch list of this bench command (`ncu --metrics
+    gpu__time_duration.sum --clock-control none`): the kernel's mean cold,
+    serialised duration and its share of the library's kernel time per update
+    (fused kernel + side-stream seal reduction), or None."""
+    try:
+        with open(os.path.join(ROOT, LAUNCH_LISTS[config])) as f:
+            t = json.load(f)
+        k = t[kernel]
+        lib = k["total_us"] + t.get("seal_reduce_kernel", {}).get("total_us", 0.0) * k["launches"] / max(
+            1, t.get("seal_reduce_kernel", {}).get("launches", 1))
+        return {"file": LAUNCH_LISTS[config], "mean_us": k["mean_us"], "share_of_library_kernels":
+                round(k["total_us"] / lib, 4), "frac_at_ncu_duration": round(alg_bytes / (k["mean_us"] * 1e3) / peak, 4)}
     except Exception:
         return None
 
@@ -140,7 +164,8 @@ def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tie
         for i in range(warmup + steps):
             v = i + 1
             G.fill_model(prod_t, specs, seed, v, stream=st)
-            G.l2_flush(flush_buf, stream=st)
+            if flush_buf is not None:  # None: warm L2 (the optimizer's writes of v are still cached)
+                G.l2_flush(flush_buf, stream=st)
             if kernel_timing:
                 torch.cuda._sleep(400_000)
             else:
@@ -382,40 +407,78 @@ def event_floor_us(G, reps=20):
     return statistics.median(out)
 
 
-def cpu_baseline(synth, name, budget_s=10.0, max_updates=100000):
-    """The oracle (plain C, single thread, as it stands) timed on this host's
-    cores on a bounded sample: repeated updates of the same config."""
-    from oracle import transfer as T
-    specs = synth.model_specs(name)
-    seed = synth.SEEDS[name]
-    nb = [synth.nbytes_of(s) for s in specs]
-    versions = [[synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)] for v in (1, 2)]
-    c = T.Consumer(nb)
-    p = T.Producer(nb, [c])
-    times = []
-    t_start = time.perf_counter()
-    v = 0
+def cpu_model():
+    """Host CPU model, the cores this process may use, and its NUMA node."""
+    model = "unknown"
     try:
+        with open("/proc/cpuinfo") as f:
+            model = next((l.split(":", 1)[1].strip() for l in f if l.startswith("model name")), model)
+    except OSError:
+        pass
+    node = None
+    try:
+        import glob
+        cpu0 = min(os.sched_getaffinity(0))
+        node = next((int(p.split("node")[-1].split("/")[0]) for p in glob.glob(f"/sys/devices/system/cpu/cpu{cpu0}/node*")),
+                    None)
+    except (OSError, ValueError):
+        pass
+    return {"model": model, "affinity_cores": len(os.sched_getaffinity(0)), "numa_node": node}
+
+
+class OracleUpdates:
+    """The oracle (plain C, single thread, as it stands) set up once for one
+    config: a producer + 1 consumer and two pre-generated versions."""
+
+    def __init__(self, synth, name):
+        from oracle import transfer as T
+        self.T, self.name = T, name
+        specs = synth.model_specs(name)
+        seed = synth.SEEDS[name]
+        nb = [synth.nbytes_of(s) for s in specs]
+        self.versions = [[synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
+                         for v in (1, 2)]
+        self.c = self.T.Consumer(nb)
+        self.p = self.T.Producer(nb, [self.c])
+        self.v = 0
+
+    def run(self, budget_s, max_updates=100000):
+        """Updates until the budget is spent; ms per update."""
+        times = []
+        t_start = time.perf_counter()
         while time.perf_counter() - t_start < budget_s and len(times) < max_updates:
-            v += 1
+            self.v += 1
             t0 = time.perf_counter()
-            st = p.publish(v, versions[v % 2])
+            st = self.p.publish(self.v, self.versions[self.v % 2])
             times.append((time.perf_counter() - t0) * 1e3)
-            assert st == T.OK
+            assert st == self.T.OK
+        return times
+
+    def close(self):
+        self.p.close()
+        self.c.close()
+
+
+def cpu_baseline(synth, name, budget_s=10.0, max_updates=100000):
+    """The oracle timed on this host's cores on a bounded sample: repeated
+    updates of the same config."""
+    o = OracleUpdates(synth, name)
+    try:
+        times = o.run(budget_s, max_updates)
     finally:
-        p.close()
-        c.close()
-    return {"value": statistics.mean(times), "unit": "ms", "cores": 1, "kind": "oracle",
+        o.close()
+    return {"value": statistics.mean(times), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
             "sample": f"{len(times)} oracle updates of {name} (pack+seal+deliver+verify+install+swap, 1 consumer)"}
 
 
 N_CONFIG = {2: "resnet50", 4: "vit_b16", 8: "gpt2_xl"}  # BASELINE.json configs[1..3]
+CONFIG_INDEX = {"ptychonn": 0, "resnet50": 1, "vit_b16": 2, "gpt2_xl": 3, "llama3_8b": 4}
 
 
 def xproc_arm(args):
     """N > 1: one process per GPU.  Rank 0 is the producer, ranks 1..N-1 the
     consumers (1 -> N-1 fan-out over NVLink: direct for one consumer,
-    scatter-allgather for more).  Each step is one SYNC update: rank 0's
+    scatter-allgather for more; --fanout chain picks the pipelined chain).  Each step is one SYNC update: rank 0's
     publish() returns once every consumer swapped.  value = mean update
     latency (host clock of rank 0 from publish entry to the last consumer's
     swap); consumers' install-kernel times (CUDA events) are
@@ -442,7 +505,10 @@ def xproc_arm(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     gloo = dist.new_group(backend="gloo")
     bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
-    fanout = V.FANOUT_SCATTER_ALLGATHER if world > 2 else V.FANOUT_DIRECT
+    fanout = {"direct": V.FANOUT_DIRECT, "chain": V.FANOUT_CHAIN, "sa": V.FANOUT_SCATTER_ALLGATHER}.get(
+        args.fanout, V.FANOUT_SCATTER_ALLGATHER if world > 2 else V.FANOUT_DIRECT)
+    fanout_name = {V.FANOUT_DIRECT: "direct pull", V.FANOUT_CHAIN: "pipelined chain",
+                   V.FANOUT_SCATTER_ALLGATHER: "scatter-allgather"}[fanout]
     role = V.PRODUCER if rank == 0 else V.CONSUMER
     m = V.Model(f"bench-x-{name}", role, tensors, fanout=fanout, flags=V.FLAG_TIMING if rank else 0,
                 device=dev, bootstrap=bs)
@@ -506,7 +572,7 @@ def xproc_arm(args):
             "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
             "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
             "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers over NVLink "
-                                   f"({'scatter-allgather' if world > 2 else 'direct pull'}), SYNC",
+                                   f"({fanout_name}), SYNC",
                        "model_bytes": S, "devices_visible": ndev,
                        "oversubscribed": ndev < world, "l2": "flushed before every update"},
             "update_gbps_per_consumer": round(S / (lat_ms * 1e-3) / 1e9, 3),
@@ -556,6 +622,7 @@ def gpu_arm(args):
         t = torch.tensor([mean_ms], device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         mean_ms = float(t.item())
+    warm = run_update_bench(V, G, synth, name, args.steps, args.warmup, None)  # cold and warm
     # kernel-only times: the fused SYNC kernel (what the headline runs) and,
     # for reference, the separate pack / install kernels (VIPER_FLAG_NO_FUSE)
     kt = run_update_bench(V, G, synth, name, args.steps, args.warmup, flush, kernel_timing=True)
@@ -574,15 +641,18 @@ def gpu_arm(args):
         "warmup": args.warmup, "ms_per_step": round(mean_ms, 6), "higher_is_better": False,
         "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
         "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
-        "config": {"workload": f"{name}: 1 producer -> 1 consumer, 1 GPU loopback (BASELINE.json configs[0])"
-                   if name == "ptychonn" else f"{name} 1-GPU loopback",
+        "config": {"workload": f"{name}: 1 producer -> 1 consumer, 1-GPU loopback "
+                               f"(BASELINE.json configs[{CONFIG_INDEX[name]}]"
+                               f"{'' if name == 'ptychonn' else ' without its NVLink hop'})",
                    "tensors": r["tensors"], "model_bytes": r["bytes"], "packed_bytes": r["s_packed"],
                    "tier": "gpu", "mode": "sync", "l2": "flushed (256 MiB write) before every timed update",
                    "parallelism": "replicas" if world > 1 else "single GPU"},
         "update_gbps": round(r["bytes"] / (mean_ms * 1e-3) / 1e9, 3),
         "host_latency_ms": round(statistics.mean(r["host_ms"]), 6),
         "latency_p50_ms": round(statistics.median(r["dev_ms"]), 6),
+        "latency_p90_ms": round(sorted(r["dev_ms"])[max(0, int(0.9 * len(r["dev_ms"]) + 0.5) - 1)], 6),
         "latency_min_ms": round(min(r["dev_ms"]), 6),
+        "latency_warm_l2_ms": round(statistics.mean(warm["dev_ms"]), 6),
         "kernels_us": {"publish_fused": round(fused, 3), "pack_seal": round(pack, 3),
                        "install_verify": round(inst, 3), "event_bracket_floor": round(calib, 3),
                        "how": "library CUDA events around each kernel, stream kept busy (no host gaps); "
@@ -591,7 +661,9 @@ def gpu_arm(args):
                      "unit": "GB/s", "frac": round(achieved / peak, 4),
                      "traffic": ncu_traffic("publish_fused_kernel", name),
                      "traffic_source": "profiles/ncu_traffic.json (ncu --set full, cold caches)",
-                     "peak_kind": peak_kind, "algorithmic_bytes": alg},
+                     "peak_kind": peak_kind, "algorithmic_bytes": alg,
+                     "duration": "CUDA events around each launch on its stream (includes the event_bracket_floor)",
+                     "ncu_launch_list": ncu_launches(name, "publish_fused_kernel", alg, peak)},
         "parity_ok": r["ok"],
         "gpu_launches": 2 * args.steps,  # publish_fused + seal_reduce per update
     }
@@ -602,7 +674,7 @@ def gpu_arm(args):
                       "d2h_bytes_per_step": e["d2h"], "digest_ok": e["ok"]}
         if not args.no_sweep:
             sweep = {}
-            for nm in ["resnet50", "vit_b16", "gpt2_xl", "llama3_8b"]:
+            for nm in ["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"]:
                 if nm == name:
                     continue
                 try:
@@ -635,7 +707,9 @@ def gpu_arm(args):
         try:
             base = {name: round(torch_copy_baseline(G, synth, name, flush), 6)}
             if not args.no_sweep:
-                for nm in ["resnet50", "vit_b16", "gpt2_xl"]:
+                for nm in ["ptychonn", "resnet50", "vit_b16", "gpt2_xl"]:
+                    if nm == name:
+                        continue
                     base[nm] = round(torch_copy_baseline(G, synth, nm, flush), 6)
             out["baseline_torch_state_dict_copy_ms"] = base
         except Exception as ex:
@@ -653,17 +727,22 @@ def reference_arm(args):
         return
     import synth
     name = args.config
+    o = OracleUpdates(synth, name)
     res = []
-    for i in range(args.warmup + args.steps):
-        cb = cpu_baseline(synth, name, budget_s=max(1.0, args.cpu_budget / max(args.steps, 1)), max_updates=20)
-        if i >= args.warmup:
-            res.append(cb["value"])
+    try:
+        for i in range(args.warmup + args.steps):
+            t = o.run(max(0.2, args.cpu_budget / max(args.steps, 1)), max_updates=20)
+            if i >= args.warmup:
+                res.append(statistics.mean(t))
+    finally:
+        o.close()
     v = statistics.mean(res)
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "ms", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(v, 4), "higher_is_better": False,
            "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
-           "data": "synthetic (VGEN)", "config": {"workload": f"{name}: oracle update on host cores"},
-           "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": 1, "kind": "oracle",
+           "data": "synthetic (VGEN)", "config": {"workload": f"{name}: 1 producer -> 1 consumer, the oracle on host cores "
+                                                     f"(BASELINE.json configs[{CONFIG_INDEX[name]}])"},
+           "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
                             "sample": "each step = up to 20 oracle updates, mean ms per update"},
            "e2e": {"value": round(v, 4), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
@@ -676,13 +755,15 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="viper", choices=["viper", "reference"])
     ap.add_argument("--config", default=None, choices=["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
+    ap.add_argument("--fanout", default="auto", choices=["auto", "direct", "chain", "sa"],
+                    help="N > 2 fan-out (auto: direct for one consumer, scatter-allgather for more)")
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     args.config_explicit = args.config is not None
     if args.config is None:
-        args.config = "ptychonn"
+        args.config = "resnet50"  # BASELINE.json configs[1] (1-GPU loopback)
     if args.impl == "reference":
         reference_arm(args)
     else:

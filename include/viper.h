@@ -94,6 +94,11 @@ enum { VIPER_TIER_GPU = 0,   /* GPU-to-GPU memory: pull over NVLink peer mapping
        VIPER_TIER_DRAM = 1 }; /* Host-to-Host memory: staged through pinned DRAM  */
 /* Fan-out of one producer to N consumers. */
 enum { VIPER_FANOUT_DIRECT = 0,        /* every consumer pulls every chunk from the producer */
+       VIPER_FANOUT_CHAIN = 1,         /* pipelined chain: consumer i pulls every item from
+                                          consumer i-1 (consumer 0 from the producer) as
+                                          soon as that item is sealed there, and stages it
+                                          for consumer i+1.  Producer egress S; bound
+                                          S/link + (N-1) items (SURVEY s8(e) option 3) */
        VIPER_FANOUT_SCATTER_ALLGATHER = 2 /* consumer i pulls chunks c = i (mod N) from the
                                              producer, the rest from its peers */ };
 /* Save mode (Fig. 3; s5.3 P:2143-2153). */

@@ -40,6 +40,9 @@ namespace {
 #ifndef VP_FUSED_BLOCKS
 #define VP_FUSED_BLOCKS 2
 #endif
+#ifndef VP_FUSED_DYNAMIC
+#define VP_FUSED_DYNAMIC 0
+#endif
 #ifndef VP_FUSED_PREFETCH
 #define VP_FUSED_PREFETCH 0  // A/B: no measurable gain (profiles/r01/ktime_prefetch_ab.log)
 #endif
@@ -339,12 +342,29 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             src = a.mp_snap[p] + it.packed_off;
             is = a.mp_iseal[p] + w;
         }
-        uint32_t owner = a.sa_n ? it.chunk % a.sa_n : 0;
-        if (a.sa_n && owner != a.sa_me) {
-            // scatter-allgather: the owner re-publishes this item in its staging
+        // Fan-out among consumers: `peer` is the consumer this item is pulled
+        // from (-1 = the producer); `republish` = also stage it (+ seal,
+        // release.sys) for the consumers that pull it from here.
+        //   scatter-allgather: chunk c is owned by consumer c % N, which pulls
+        //                      it from the producer; the others pull from it;
+        //   chain:             consumer i pulls everything from consumer i-1
+        //                      (0 from the producer) and stages it for i+1.
+        int peer = -1;
+        bool republish = false;
+        if (a.sa_n) {
+            if (a.chain) {
+                peer = (int)a.sa_me - 1;
+                republish = a.sa_me + 1 < a.sa_n;
+            } else if (it.chunk % a.sa_n == a.sa_me) {
+                republish = true;
+            } else {
+                peer = (int)(it.chunk % a.sa_n);
+            }
+        }
+        if (peer >= 0) {
             int ok = 0;
             if (lane == 0) {
-                const ISeal *ps = a.sa_isrc[owner] + w;
+                const ISeal *ps = a.sa_isrc[peer] + w;
                 uint32_t backoff = 64;
                 int64_t spent = 0;
                 for (;;) {
@@ -352,18 +372,18 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                     __nanosleep(backoff);
                     spent += backoff;
                     if (backoff < 2048) backoff <<= 1;
-                    // the owner is not installing this version (skipped it or
+                    // the peer is not installing this version (skipped it or
                     // finished without it): take the item from the producer
-                    if (spent > 20000 && *a.sa_owner_pin[owner] != a.version) break;
+                    if (spent > 20000 && *a.sa_owner_pin[peer] != a.version) break;
                     if (spent > 50000000) break;  // 50 ms: never hang, fall back
                 }
             }
             ok = __shfl_sync(0xffffffffu, ok, 0);
             if (ok) {
-                src = a.sa_src[owner] + it.packed_off;
-                is = a.sa_isrc[owner] + w;
+                src = a.sa_src[peer] + it.packed_off;
+                is = a.sa_isrc[peer] + w;
             } else {
-                owner = a.sa_me;  // producer copy; not re-published
+                peer = -1;  // producer copy (re-published only where this consumer stages it anyway)
             }
         }
         // (system scope: the producer may be another GPU pipelining its pack)
@@ -383,15 +403,26 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             expect = is->mixed;
         }
         __syncwarp();
-        const bool republish = a.sa_n && owner == a.sa_me && it.chunk % a.sa_n == a.sa_me;
+        const bool from_peer = peer >= 0;
         if (republish) {
             // src -> slot, then the slot bytes just stored are read back into
             // this consumer's staging (what its peers will pull)
             uint64_t dsts[kMaxFused] = {(uint64_t)(a.sa_stage_out + it.packed_off), 0, 0, 0};
             uint64_t got[kMaxFused] = {0, 0, 0, 0};
-            const uint64_t part = warp_sum(copy_item_fused(src, (uint8_t *)it.ptr, dsts, 1, it.nbytes, it.packed_off,
-                                                           lane, w == a.fault_item ? 1u : 0u, got));
-            const uint64_t staged = warp_sum(got[0]);
+            uint64_t part = warp_sum(copy_item_fused(src, (uint8_t *)it.ptr, dsts, 1, it.nbytes, it.packed_off,
+                                                     lane, w == a.fault_item ? 1u : 0u, got));
+            uint64_t staged = warp_sum(got[0]);
+            // chain: the predecessor's staged copy failed its seal -> heal from
+            // the producer (pinned by this consumer) before staging it onward
+            if (__shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0)) {
+                const ISeal *ps = a.iseal + w;
+                const uint64_t pexp = lane == 0 ? ps->mixed : 0;
+                got[0] = 0;
+                part = warp_sum(copy_item_fused(a.packed + it.packed_off, (uint8_t *)it.ptr, dsts, 1, it.nbytes,
+                                                it.packed_off, lane, 0u, got));
+                staged = warp_sum(got[0]);
+                if (lane == 0) expect = pexp;
+            }
             __syncwarp();
             if (lane == 0) {  // peers may now pull item w from this consumer's staging
                 a.sa_iseal_out[w].mixed = expect;
@@ -401,7 +432,6 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
         } else {
             uint64_t part = warp_sum(
                 copy_item<true>(src, (uint8_t *)it.ptr, it.nbytes, it.packed_off, lane, w == a.fault_item));
-            const bool from_peer = a.sa_n && owner != a.sa_me;
             // expect is valid in lane 0 only: take the (warp-uniform) decision there
             const int heal = __shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0);
             if (heal) {
@@ -428,11 +458,24 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+#if VP_FUSED_DYNAMIC
+    // first round static, then items handed out by a counter (balances the
+    // tail: item sizes differ at tensor borders); the next index is claimed
+    // while the current item streams
+    unsigned int *ctr = reinterpret_cast<unsigned int *>(a.flags + 1);
+    uint32_t nxt_w = 0;
+    if (lane == 0 && w < a.nitems) nxt_w = nwarps + atomicAdd(ctr, 1u);
+    nxt_w = __shfl_sync(0xffffffffu, nxt_w, 0);
+#endif
 #if VP_FUSED_PREFETCH
     Item nxt{};
     if (w < a.nitems) nxt = a.items[w];
 #endif
+#if VP_FUSED_DYNAMIC
+    for (; w < a.nitems;) {
+#else
     for (; w < a.nitems; w += nwarps) {
+#endif
 #if VP_FUSED_PREFETCH
         const Item it = nxt;  // descriptor prefetched one item ahead
         if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
@@ -459,11 +502,19 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
             if (k >= (int)a.ncons) break;
             if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
         }
+#if VP_FUSED_DYNAMIC
+        w = nxt_w;
+        if (lane == 0 && w < a.nitems) nxt_w = nwarps + atomicAdd(ctr, 1u);
+        nxt_w = __shfl_sync(0xffffffffu, nxt_w, 0);
+#endif
     }
     if (lane == 0 && bad) report_err(a.flags, bad);
     __syncthreads();
     uint32_t e;
     if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
+#if VP_FUSED_DYNAMIC
+        *reinterpret_cast<unsigned int *>(a.flags + 1) = 0;  // every warp stopped claiming
+#endif
         for (uint32_t k = 0; k < a.ncons; k++) {
             const FusedCons &c = a.cons[k];
             const int32_t st = (e >> k) & 1u ? -5 : 0;

@@ -1018,7 +1018,8 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
         if (c.chunk_bytes % 256 || c.chunk_bytes % c.align) return set_error(VIPER_E_INVAL, "chunk_bytes must be a multiple of 256 and align");
         if (c.tier != VIPER_TIER_GPU && c.tier != VIPER_TIER_DRAM) return set_error(VIPER_E_INVAL, "bad tier");
         if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
-        if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER)
+        if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_CHAIN &&
+            c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER)
             return set_error(VIPER_E_UNSUPPORTED, "fanout %d not supported", c.fanout);
         int ndev = 0;
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0)

@@ -83,7 +83,10 @@ struct InstallArgs {
     // peers; the others are pulled from the owner's staging once its seal
     // shows `version`, falling back to the producer when the owner is not
     // installing this version.
-    uint32_t sa_n, sa_me;
+    // Chain fan-out (sa_n > 0, chain = 1): consumer i pulls every item from
+    // consumer i-1's staging (consumer 0 from the producer) and stages it for
+    // consumer i+1 (all but the last), with the same seals and fallbacks.
+    uint32_t sa_n, sa_me, chain;
     // Multi-producer fan-in (mp_n > 1): item x comes from producer
     // chunk(x) % mp_n (data-parallel replicas each pack their share)
     uint32_t mp_n;

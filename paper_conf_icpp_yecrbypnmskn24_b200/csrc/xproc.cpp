@@ -286,9 +286,11 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
         }
     }
-    const bool sa = m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER;
+    // consumers stage what their peers pull from them: the chunks they own
+    // (scatter-allgather) or everything (chain)
+    const bool sa = m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER || m->cfg.fanout == VIPER_FANOUT_CHAIN;
     if (st == VIPER_OK && !producer && sa) {
-        // my staging for the chunks I own, double-buffered by snapshot slot
+        // my staging, double-buffered by snapshot slot
         m->sa_S = S;
         m->sa_IS = IS;
         cudaError_t e = cudaMalloc(&m->sa_alloc, 2 * (S + IS));
@@ -399,7 +401,9 @@ viper_status xproc_install(viper_model *c, uint64_t v, int b) {
         pi.a.mp_iseal = (const ISeal *const *)(tab + 2 * M + b * M);
         return launch_prepared(pi, c->xsrc, b, c->ustream, false, false);
     }
-    if (c->cfg.fanout != VIPER_FANOUT_SCATTER_ALLGATHER || c->nconsumers_x < 2 || c->cfg.tier != VIPER_TIER_GPU)
+    const bool chain = c->cfg.fanout == VIPER_FANOUT_CHAIN;
+    if ((c->cfg.fanout != VIPER_FANOUT_SCATTER_ALLGATHER && !chain) || c->nconsumers_x < 2 ||
+        c->cfg.tier != VIPER_TIER_GPU)
         return enqueue_install(c, c->xsrc, v, b, c->ustream, false);
     PreparedInstall pi;
     viper_status s = prepare_install(c, c->xsrc, v, b, &pi);
@@ -408,6 +412,7 @@ viper_status xproc_install(viper_model *c, uint64_t v, int b) {
     const void *const *tab = (const void *const *)c->d_sa_tab;
     pi.a.sa_n = (uint32_t)N;
     pi.a.sa_me = (uint32_t)c->cidx;
+    pi.a.chain = chain ? 1u : 0u;
     pi.a.sa_stage_out = (uint8_t *)c->sa_alloc + b * c->sa_S;
     pi.a.sa_iseal_out = (ISeal *)((uint8_t *)c->sa_alloc + 2 * c->sa_S + b * c->sa_IS);
     pi.a.sa_src = (const uint8_t *const *)(tab + b * N);

@@ -17,7 +17,7 @@ OK, E_INVAL, E_NOMEM, E_CUDA, E_VERSION, E_CHECKSUM, E_TIMEOUT, E_NOVERSION, E_S
 PRODUCER, CONSUMER = 1, 2
 F32, BF16, F16, BYTES = 0, 1, 2, 3
 TIER_GPU, TIER_DRAM = 0, 1
-FANOUT_DIRECT, FANOUT_SCATTER_ALLGATHER = 0, 2
+FANOUT_DIRECT, FANOUT_CHAIN, FANOUT_SCATTER_ALLGATHER = 0, 1, 2
 SYNC, ASYNC = 0, 1
 FLAG_TIMING = 2
 FLAG_NO_FUSE = 4

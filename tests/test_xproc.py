@@ -58,7 +58,28 @@ def test_xproc_scatter_allgather_fault():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("nproc,fanout,mode", [(2, 0, 0), (3, 0, 1), (4, 2, 0)])
+@pytest.mark.parametrize("nproc,mode,config", [(3, 0, "ptychonn"), (4, 0, "small"), (4, 1, "small"),
+                                              (5, 0, "resnet50")])
+def test_xproc_chain(nproc, mode, config):
+    """Pipelined chain fan-out (SURVEY s8(e) option 3): consumer i pulls every
+    item from consumer i-1's staging, verifies it and stages it for i+1."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", config, "--mode", str(mode), "--fanout", "1", "--versions", "5"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+def test_xproc_chain_fault():
+    """A flipped bit in one chain link's copy: that consumer reports
+    VIPER_E_CHECKSUM and keeps serving the previous version (the worker checks
+    it); its successor heals from the producer."""
+    rc, out = run_torchrun(4, "tests/xproc_worker.py", ["--config", "small", "--fanout", "1", "--fault", "1",
+                                                       "--versions", "3"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,fanout,mode", [(2, 0, 0), (3, 0, 1), (4, 2, 0), (4, 1, 0), (3, 1, 1)])
 def test_xproc_early_notify_pipeline(nproc, fanout, mode):
     """Cross-GPU item pipeline: v is published right after the pack launch and
     consumers' install kernels wait per item on seals released at system scope
@@ -81,7 +102,7 @@ def test_xproc_early_notify_waits_for_the_stream():
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("nproc,fanout", [(3, 0), (4, 2)])
+@pytest.mark.parametrize("nproc,fanout", [(3, 0), (4, 2), (4, 1)])
 def test_xproc_no_torn_reads(nproc, fanout):
     rc, out = run_torchrun(nproc, "tests/xproc_worker.py", ["--config", "small", "--mode", "1", "--fanout",
                                                            str(fanout), "--stress", "1", "--versions", "200"])
