@@ -40,6 +40,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+HBM_NOMINAL_GBS = 7700.0  # B200 HGX HBM3e nominal (B200_PROFILING.md), context beside the measured copy peak
 METRIC = "model-update latency (ms) and GB/s vs NVLink/HBM roofline at 1->1/3/7 GPUs"
 
 
@@ -663,7 +664,8 @@ def gpu_arm(args):
                      "traffic_source": "profiles/ncu_traffic.json (ncu --set full, cold caches)",
                      "peak_kind": peak_kind, "algorithmic_bytes": alg,
                      "duration": "CUDA events around each launch on its stream (includes the event_bracket_floor)",
-                     "ncu_launch_list": ncu_launches(name, "publish_fused_kernel", alg, peak)},
+                     "ncu_launch_list": ncu_launches(name, "publish_fused_kernel", alg, peak),
+                     "frac_of_nominal_7700": round(achieved / HBM_NOMINAL_GBS, 4)},
         "parity_ok": r["ok"],
         "gpu_launches": 2 * args.steps,  # publish_fused + seal_reduce per update
     }
@@ -688,6 +690,8 @@ def gpu_arm(args):
                     sweep[nm] = {"latency_ms": round(lat, 4), "fused_us": round(fu, 2), "pack_us": round(pk, 2),
                                  "install_us": round(ins, 2),
                                  "fused_hbm_frac": round(3 * s["bytes"] / (fu * 1e-6) / 1e9 / peak, 4),
+                                 "fused_frac_of_nominal_7700": round(3 * s["bytes"] / (fu * 1e-6) / 1e9 /
+                                                                     HBM_NOMINAL_GBS, 4),
                                  "pack_hbm_frac": round(2 * s["bytes"] / (pk * 1e-6) / 1e9 / peak, 4),
                                  "install_hbm_frac": round(2 * s["bytes"] / (ins * 1e-6) / 1e9 / peak, 4),
                                  "update_gbps": round(s["bytes"] / (lat * 1e-3) / 1e9, 2),

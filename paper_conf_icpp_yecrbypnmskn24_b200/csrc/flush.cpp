@@ -282,6 +282,7 @@ extern "C" viper_status viper_restore(const char *path, const viper_tensor *tens
             a.version = hd.version;
             a.fault_item = ~0u;
             a.flags = (unsigned long long *)flags;
+            a.ctr = (unsigned int *)((uint8_t *)flags + 8);  // zeroed above
             a.status_h = (volatile int32_t *)sh_dev;
             e = launch_install(a, pick_geometry(a.nitems, device), s, false);
         }

@@ -40,11 +40,8 @@ namespace {
 #ifndef VP_FUSED_BLOCKS
 #define VP_FUSED_BLOCKS 2
 #endif
-#ifndef VP_FUSED_DYNAMIC
-#define VP_FUSED_DYNAMIC 0
-#endif
-#ifndef VP_FUSED_PREFETCH
-#define VP_FUSED_PREFETCH 0  // A/B: no measurable gain (profiles/r01/ktime_prefetch_ab.log)
+#ifndef VP_DYNAMIC
+#define VP_DYNAMIC 1  // A/B: profiles/r01/ktime_dynamic_ab.log
 #endif
 constexpr int kWarpsPerBlock = VP_WARPS_PER_BLOCK;  // 256 threads
 constexpr int kBlocksPerSM = VP_BLOCKS_PER_SM;      // 512 threads / SM resident (128-reg budget)
@@ -107,6 +104,32 @@ __device__ __forceinline__ uint64_t warp_sum(uint64_t x) {
     for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
     return x;
 }
+
+// Work distribution of the streaming kernels.  Each warp's first item is
+// static (its global warp id); after that, items are claimed from a per-launch
+// counter, one item ahead, so the atomic's round trip overlaps the current
+// item's stream.  This balances the tail (item sizes differ at tensor and
+// chunk borders, SMs progress at different rates).  Claimed index = raw -
+// base + nwarps; the grid's last block resets the counter (base 0).  With
+// nitems <= nwarps there is no second round and no claim.  Used by the fused
+// and install kernels; the pack stays static (measured faster, see there).
+struct WorkQueue {
+    unsigned int *ctr;
+    uint32_t base, nwarps, nitems;
+    bool dyn;
+    uint32_t pending;  // lane 0: raw value of the claim in flight
+    __device__ __forceinline__ WorkQueue(unsigned int *c, uint32_t b, uint32_t nw, uint32_t n)
+        : ctr(c), base(b), nwarps(nw), nitems(n), dyn(VP_DYNAMIC && c != nullptr && n > nw), pending(0) {}
+    __device__ __forceinline__ void claim(uint32_t lane) {
+        if (dyn && lane == 0) pending = atomicAdd(ctr, 1u);
+    }
+    // the item after w: the claim made one item ago (or the static stride)
+    __device__ __forceinline__ uint32_t next(uint32_t w, uint32_t lane) {
+        if (!dyn) return w + nwarps;
+        const uint32_t k = __shfl_sync(0xffffffffu, pending - base, 0);
+        return k < nitems ? k + nwarps : nitems;  // k >= nitems: wrapped / exhausted
+    }
+};
 
 // Copy bytes [b0, n) of an item word by word (any alignment); words are
 // little-endian u32 of the packed buffer, zero-extended past n.
@@ -246,6 +269,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
     asm volatile("griddepcontrol.launch_dependents;");
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    // Static strided items: measured faster than the work counter here
+    // (Llama-3 8B 5.05 vs 6.0 ms, profiles/r01/ktime_dynamic_ab.log).
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     Item nxt{};
     if (w < a.nitems) nxt = a.items[w];
@@ -316,6 +341,7 @@ __device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
         if (a.status_h) *a.status_h = st;
         if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
         if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
+        if (a.ctr) *a.ctr = 0;      // work counter: every warp stopped claiming
     }
 }
 
@@ -327,10 +353,10 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     bool bad = false;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
-    Item it{};
-    if (w < a.nitems) it = a.items[w];
-    for (; w < a.nitems; w += nwarps) {
-        if (w >= blockIdx.x * kWarpsPerBlock + nwarps) it = a.items[w];
+    WorkQueue q(a.ctr, 0, nwarps, a.nitems);  // reset by the last block (install_finish)
+    if (w < a.nitems) q.claim(lane);
+    while (w < a.nitems) {
+        const Item it = a.items[w];
         // Item-granular pipeline: with PDL the install grid runs concurrently
         // with the pack grid (all of whose blocks are resident by then, so
         // this cannot deadlock); wait for item w's ready flag, then stream it
@@ -403,48 +429,44 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             expect = is->mixed;
         }
         __syncwarp();
-        const bool from_peer = peer >= 0;
-        if (republish) {
-            // src -> slot, then the slot bytes just stored are read back into
-            // this consumer's staging (what its peers will pull)
-            uint64_t dsts[kMaxFused] = {(uint64_t)(a.sa_stage_out + it.packed_off), 0, 0, 0};
-            uint64_t got[kMaxFused] = {0, 0, 0, 0};
-            uint64_t part = warp_sum(copy_item_fused(src, (uint8_t *)it.ptr, dsts, 1, it.nbytes, it.packed_off,
-                                                     lane, w == a.fault_item ? 1u : 0u, got));
-            uint64_t staged = warp_sum(got[0]);
-            // chain: the predecessor's staged copy failed its seal -> heal from
-            // the producer (pinned by this consumer) before staging it onward
-            if (__shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0)) {
-                const ISeal *ps = a.iseal + w;
-                const uint64_t pexp = lane == 0 ? ps->mixed : 0;
-                got[0] = 0;
-                part = warp_sum(copy_item_fused(a.packed + it.packed_off, (uint8_t *)it.ptr, dsts, 1, it.nbytes,
-                                                it.packed_off, lane, 0u, got));
+        // One pass, or two when a peer's staged copy failed its seal: the
+        // second pass heals from the producer (pinned by this consumer) and
+        // verifies against the producer's own seal.  (A loop, not a second
+        // inlined copy: the kernel stays within its 128-register budget.)
+        bool from_peer = peer >= 0;
+        for (;;) {
+            uint64_t part, staged = 0;
+            if (republish) {
+                // src -> slot, then the slot bytes just stored are read back
+                // into this consumer's staging (what its peers will pull)
+                uint64_t dsts[kMaxFused] = {(uint64_t)(a.sa_stage_out + it.packed_off), 0, 0, 0};
+                uint64_t got[kMaxFused] = {0, 0, 0, 0};
+                part = warp_sum(copy_item_fused(src, (uint8_t *)it.ptr, dsts, 1, it.nbytes, it.packed_off, lane,
+                                                w == a.fault_item ? 1u : 0u, got));
                 staged = warp_sum(got[0]);
-                if (lane == 0) expect = pexp;
+            } else {
+                part = warp_sum(copy_item<true>(src, (uint8_t *)it.ptr, it.nbytes, it.packed_off, lane,
+                                                w == a.fault_item));  // injected on every pass: never healed
             }
-            __syncwarp();
-            if (lane == 0) {  // peers may now pull item w from this consumer's staging
-                a.sa_iseal_out[w].mixed = expect;
-                st_release_sys(&a.sa_iseal_out[w].version, a.version);
-                if (part + a.version * kVerMix != expect || staged + a.version * kVerMix != expect) bad = true;
-            }
-        } else {
-            uint64_t part = warp_sum(
-                copy_item<true>(src, (uint8_t *)it.ptr, it.nbytes, it.packed_off, lane, w == a.fault_item));
             // expect is valid in lane 0 only: take the (warp-uniform) decision there
-            const int heal = __shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0);
-            if (heal) {
-                // a peer's staged copy failed its seal: heal from the producer
-                // (pinned by this consumer) and verify against its own seal
-                const ISeal *ps = a.iseal + w;
-                const uint64_t pexp = lane == 0 ? ps->mixed : 0;
-                part = warp_sum(copy_item<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes,
-                                                it.packed_off, lane, false));
-                if (lane == 0) expect = pexp;
+            if (__shfl_sync(0xffffffffu, (int)(from_peer && part + a.version * kVerMix != expect), 0)) {
+                src = a.packed + it.packed_off;
+                if (lane == 0) expect = a.iseal[w].mixed;
+                from_peer = false;
+                continue;
             }
-            if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
+            if (lane == 0) {
+                if (republish) {  // peers may now pull item w from this consumer's staging
+                    a.sa_iseal_out[w].mixed = expect;
+                    st_release_sys(&a.sa_iseal_out[w].version, a.version);
+                    if (staged + a.version * kVerMix != expect) bad = true;
+                }
+                if (part + a.version * kVerMix != expect) bad = true;
+            }
+            break;
         }
+        w = q.next(w, lane);
+        if (w < a.nitems) q.claim(lane);
     }
     install_finish(a, bad);
 }
@@ -458,30 +480,10 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
-#if VP_FUSED_DYNAMIC
-    // first round static, then items handed out by a counter (balances the
-    // tail: item sizes differ at tensor borders); the next index is claimed
-    // while the current item streams
-    unsigned int *ctr = reinterpret_cast<unsigned int *>(a.flags + 1);
-    uint32_t nxt_w = 0;
-    if (lane == 0 && w < a.nitems) nxt_w = nwarps + atomicAdd(ctr, 1u);
-    nxt_w = __shfl_sync(0xffffffffu, nxt_w, 0);
-#endif
-#if VP_FUSED_PREFETCH
-    Item nxt{};
-    if (w < a.nitems) nxt = a.items[w];
-#endif
-#if VP_FUSED_DYNAMIC
-    for (; w < a.nitems;) {
-#else
-    for (; w < a.nitems; w += nwarps) {
-#endif
-#if VP_FUSED_PREFETCH
-        const Item it = nxt;  // descriptor prefetched one item ahead
-        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
-#else
+    WorkQueue q(reinterpret_cast<unsigned int *>(a.flags + 1), 0, nwarps, a.nitems);  // reset by the last block
+    if (w < a.nitems) q.claim(lane);
+    while (w < a.nitems) {
         const Item it = a.items[w];
-#endif
         uint64_t cptr[kMaxFused];  // only the slot address differs between the lists
         uint32_t inject = 0;
 #pragma unroll
@@ -502,19 +504,14 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
             if (k >= (int)a.ncons) break;
             if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
         }
-#if VP_FUSED_DYNAMIC
-        w = nxt_w;
-        if (lane == 0 && w < a.nitems) nxt_w = nwarps + atomicAdd(ctr, 1u);
-        nxt_w = __shfl_sync(0xffffffffu, nxt_w, 0);
-#endif
+        w = q.next(w, lane);
+        if (w < a.nitems) q.claim(lane);
     }
     if (lane == 0 && bad) report_err(a.flags, bad);
     __syncthreads();
     uint32_t e;
     if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
-#if VP_FUSED_DYNAMIC
-        *reinterpret_cast<unsigned int *>(a.flags + 1) = 0;  // every warp stopped claiming
-#endif
+        *reinterpret_cast<unsigned int *>(a.flags + 1) = 0;  // work counter: every warp stopped claiming
         for (uint32_t k = 0; k < a.ncons; k++) {
             const FusedCons &c = a.cons[k];
             const int32_t st = (e >> k) & 1u ? -5 : 0;

@@ -347,6 +347,7 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
     a.fault_item = ~0u;
     if (c->fault_next.exchange(false) && a.nitems) a.fault_item = a.nitems / 2;
     a.flags = (unsigned long long *)c->d_flags;
+    a.ctr = (unsigned int *)((uint8_t *)c->d_flags + 8);  // [8, 12): the install's work counter
     a.status_h = (volatile int32_t *)&c->rec_dev->status;
     a.pin_h = (volatile uint64_t *)&c->rec_dev->pin;
     a.state_h = (volatile uint64_t *)&c->rec_dev->state;

@@ -112,7 +112,8 @@ struct viper_model {
     viper_config cfg{};
     vp::Manifest man;
     vp::Geometry geo{};
-    uint32_t *d_flags = nullptr;       // consumer: [0] done blocks, [1] error bits
+    uint32_t *d_flags = nullptr;       // 64 B: [0, 8) grid completion (blocks | error bits), [8, 12) install / fused
+                                       // work counter (kernels.cu WorkQueue)
     vp::Channel *chan = nullptr;       // in-process channel (registry entry)
     vp::Ctrl *ctrl = nullptr;          // host view of the control block
     vp::Ctrl *ctrl_dev = nullptr;      // device view (mapped)

@@ -71,6 +71,7 @@ struct InstallArgs {
     uint32_t target;            // slot being written
     uint32_t fault_item;        // item whose first word is flipped (fault injection); ~0u = none
     unsigned long long *flags;  // [1] low 32 bits: blocks finished; high 32: error bits (self-resetting)
+    unsigned int *ctr;          // work counter (kernels.cu WorkQueue), reset by the last block; NULL = static
     // Host-mapped control words (cudaHostAlloc/cudaHostRegister mapped).  The
     // last block writes *status_h, clears *pin_h and, when every item matched,
     // flips *state_h = (version << 1) | target: the atomic version swap.
@@ -118,7 +119,8 @@ struct FusedArgs {
     uint8_t *packed;
     ISeal *iseal;
     uint64_t version;
-    unsigned long long *flags;  // [1] low 32: blocks finished; high 32: bit k = consumer k failed (self-resetting)
+    unsigned long long *flags;  // [1] low 32: blocks finished; high 32: bit k = consumer k failed (self-resetting);
+                                // flags + 1: the work counter (kernels.cu WorkQueue), reset by the last block
     FusedCons cons[kMaxFused];
 };
 

@@ -353,7 +353,11 @@ def test_no_torn_reads_under_async_publishes():
 @pytest.mark.parametrize("name,flags,tier", [("resnet50", 0, V.TIER_GPU), ("vit_b16", 0, V.TIER_GPU),
                                              ("gpt2_xl", 0, V.TIER_GPU), ("llama3_8b", 0, V.TIER_GPU),
                                              ("gpt2_xl", V.FLAG_TMA, V.TIER_GPU), ("resnet50", 0, V.TIER_DRAM),
-                                             ("gpt2_xl", 0, V.TIER_DRAM)])
+                                             ("gpt2_xl", 0, V.TIER_DRAM),
+                                             # register pack + PDL register install: > one round of items per
+                                             # warp, so both work counters hand out items (kernels.cu WorkQueue)
+                                             ("resnet50", V.FLAG_NO_FUSE, V.TIER_GPU),
+                                             ("vit_b16", V.FLAG_NO_FUSE | V.FLAG_NO_TMA, V.TIER_GPU)])
 def test_full_size_loopback_sampled(name, flags, tier):
     """Full BASELINE.json model sizes, single-GPU loopback (the launch config
     bench.py times): every seal's version; sampled chunk seals recomputed by the
