@@ -255,13 +255,17 @@ def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
     return {"ms": statistics.mean(times), "h2d": flat.numel(), "d2h": 16 * nchunks, "ok": ok}
 
 
-def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
+def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0, install_sms=0, reader_kind="verify"):
     """BASELINE.json configs[2] in 1-GPU loopback: ViT-B/16 bf16 consumer serving
     while ASYNC updates land.  A reader thread loops acquire -> read every weight
     byte and compare with VGEN(view.version) on the GPU (a bandwidth-heavy
     stand-in for inference) -> stream-ordered release.  Reports
     verified views/s without and with publishes every `period_ms`, torn views
-    (must be 0) and the install latency seen by the consumer."""
+    (must be 0) and the install latency seen by the consumer.
+    reader_kind="gemm": a compute-bound stand-in instead -- per view, the 48
+    linear layers of the 12 encoder blocks (in_proj, out_proj, mlp.0, mlp.3,
+    bf16 tensor cores) over a batch of 64 images x 197 tokens, using the
+    view's weights."""
     import threading
     import torch
     name = "vit_b16"
@@ -269,7 +273,7 @@ def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
     seed = synth.SEEDS[name]
     pt, ct = G.alloc_model(specs), G.alloc_model(specs)
     mname = f"c3-{os.getpid()}-{time.monotonic_ns()}"
-    cons = V.Model(mname, V.CONSUMER, ct)
+    cons = V.Model(mname, V.CONSUMER, ct, install_sms=install_sms)
     prod = V.Model(mname, V.PRODUCER, pt, mode=V.ASYNC)
     G.fill_model(pt, specs, seed, 1)
     prod.publish(1)
@@ -282,8 +286,20 @@ def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
         s = torch.cuda.Stream()
         exp = G.alloc_model(specs)
         last = 0
+        lin = [i for i, sp in enumerate(specs) if len(sp[2]) == 2 and sp[2][1] in (768, 3072) and "encoder" in sp[0]]
+        x0 = torch.randn(64 * 197, 768, dtype=torch.bfloat16, device="cuda") if reader_kind == "gemm" else None
         with torch.cuda.stream(s):
-            while not stop.is_set():
+            while not stop.is_set() and reader_kind == "gemm":
+                view = cons.acquire_latest(timeout_us=100_000)
+                w = view.tensors(ct)
+                x = x0
+                for i in lin:  # x @ W^T through the encoder's linear layers (shapes chain per block)
+                    y = x @ w[i].t()
+                    x = y[:, :768] if y.shape[1] == 2304 else y
+                cons.release(view, stream=s)
+                s.synchronize()
+                stats["views"] += 1
+            while not stop.is_set() and reader_kind == "verify":
                 view = cons.acquire_latest(timeout_us=100_000)
                 G.fill_model(exp, specs, seed, view.version, stream=s)
                 bad = torch.zeros((), dtype=torch.int64, device="cuda")
@@ -326,7 +342,9 @@ def c3_concurrent(V, G, synth, seconds=1.5, period_ms=2.0):
         cons.close()
         prod.close()
     return {"workload": "vit_b16 bf16 1 producer -> 1 consumer (1-GPU loopback), ASYNC, publish every "
-                        f"{period_ms} ms", "reader": "acquire -> byte-compare every weight with VGEN -> release",
+                        f"{period_ms} ms", "install_sms": install_sms or "all", "reader_kind": reader_kind,
+            "reader": "acquire -> byte-compare every weight with VGEN -> release" if reader_kind == "verify" else
+                      "acquire -> 48 encoder linears (bf16 GEMMs, 64 x 197 tokens) on the view's weights -> release",
             "views_per_s_idle": round(base, 1), "views_per_s_during_updates": round(busy, 1),
             "throughput_drop": round(1 - busy / base, 4) if base else None, "publishes": npub,
             "installs": cst["installs"], "skipped": cst["skipped"], "torn_views": stats["torn"],
@@ -702,6 +720,7 @@ def gpu_arm(args):
             out["loopback_sweep"] = sweep
             try:
                 out["c3_concurrent"] = c3_concurrent(V, G, synth)
+                out["c3_concurrent_gemm"] = c3_concurrent(V, G, synth, reader_kind="gemm")  # compute-bound reader
             except Exception as ex:
                 out["c3_concurrent"] = {"error": str(ex)[:200]}
             try:

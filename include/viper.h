@@ -138,6 +138,13 @@ typedef struct {
                                 background thread").  Pinned double
                                 buffer; a version is skipped (counted) when storage
                                 is behind.  NULL = off.  Not with nproducers > 1.  */
+    int32_t install_sms;     /* consumer: run its install kernel on at most this many SMs
+                                (0 = all).  Bounds an update's share of the GPU while the
+                                replica serves ("inference continues"): the
+                                install takes longer, the other SMs stay with inference.
+                                Applies to the consumer's own install kernel (ASYNC, DRAM
+                                tier, cross-process), not to a SYNC in-process publish,
+                                which installs inside the producer's fused kernel.     */
 } viper_config;
 
 typedef struct viper_model viper_model; /* opaque */

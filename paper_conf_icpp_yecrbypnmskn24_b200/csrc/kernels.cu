@@ -780,7 +780,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
 
 }  // namespace
 
-Geometry pick_geometry(uint32_t nitems, int device) {
+Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
     static int sms = 0;
     if (sms == 0) {
         if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) sms = 148;
@@ -789,7 +789,7 @@ Geometry pick_geometry(uint32_t nitems, int device) {
     g.items = nitems;
     g.block = kWarpsPerBlock * 32;
     const uint32_t want = (nitems + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    const uint32_t cap = (uint32_t)sms * kBlocksPerSM;
+    const uint32_t cap = (uint32_t)(max_sms > 0 && max_sms < sms ? max_sms : sms) * kBlocksPerSM;
     g.grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
     return g;
 }
@@ -834,7 +834,7 @@ cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st)
     return cudaGetLastError();
 }
 
-cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device) {
+cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device, int max_sms) {
     static int sms = 0;
     const size_t smem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
     if (sms == 0) {
@@ -844,7 +844,7 @@ cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device
         if (e != cudaSuccess) return e;
     }
     const uint32_t want = (a.nitems + kTmaWarps - 1) / kTmaWarps;
-    const uint32_t cap = (uint32_t)sms * 2;
+    const uint32_t cap = (uint32_t)(max_sms > 0 && max_sms < sms ? max_sms : sms) * 2;
     const int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
     install_verify_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
     return cudaGetLastError();

@@ -387,7 +387,7 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     const bool tma = direct && complete && !(c->cfg.flags & VIPER_FLAG_NO_TMA) &&
                      ((c->cfg.flags & VIPER_FLAG_TMA) || c->man.s_packed <= (1ull << 30));
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
-    if (tma) CUDA_TRY(launch_install_tma(pi.a, st, c->device));
+    if (tma) CUDA_TRY(launch_install_tma(pi.a, st, c->device, c->cfg.install_sms));
     else CUDA_TRY(launch_install(pi.a, c->geo, st, pdl && !timing));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
@@ -1019,6 +1019,7 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
         if (c.chunk_bytes % 256 || c.chunk_bytes % c.align) return set_error(VIPER_E_INVAL, "chunk_bytes must be a multiple of 256 and align");
         if (c.tier != VIPER_TIER_GPU && c.tier != VIPER_TIER_DRAM) return set_error(VIPER_E_INVAL, "bad tier");
         if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
+        if (c.install_sms < 0) return set_error(VIPER_E_INVAL, "install_sms must be >= 0");
         if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_CHAIN &&
             c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER)
             return set_error(VIPER_E_UNSUPPORTED, "fanout %d not supported", c.fanout);
@@ -1036,7 +1037,8 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
         m->cfg = c;
         st = build_manifest(m->man, tensors, n, c.chunk_bytes, c.align, c.device);
         if (!st) {
-            m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device);
+            m->geo = pick_geometry((uint32_t)m->man.items.size(), c.device,
+                                   role == VIPER_CONSUMER ? c.install_sms : 0);
             if (bs && bs->world > 1) {
                 m->xproc = true;
                 *joined = true;

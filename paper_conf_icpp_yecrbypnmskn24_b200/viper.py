@@ -42,7 +42,7 @@ class viper_bootstrap(C.Structure):
 class viper_config(C.Structure):
     _fields_ = [("tier", C.c_int32), ("fanout", C.c_int32), ("mode", C.c_int32), ("chunk_bytes", C.c_uint64),
                 ("align", C.c_uint32), ("device", C.c_int32), ("slot1", C.POINTER(viper_tensor)),
-                ("flags", C.c_int32), ("flush_dir", C.c_char_p)]
+                ("flags", C.c_int32), ("flush_dir", C.c_char_p), ("install_sms", C.c_int32)]
 
 
 class viper_view(C.Structure):
@@ -210,7 +210,7 @@ class Model:
 
     def __init__(self, name: str, role: int, tensors, *, tier=TIER_GPU, fanout=FANOUT_DIRECT, mode=SYNC,
                  chunk_bytes=0, align=0, device=None, slot1=None, flags=0, bootstrap=None, names=None,
-                 flush_dir=None):
+                 flush_dir=None, install_sms=0):
         L = lib()
         self.tensors = list(tensors)
         self.role = role
@@ -218,7 +218,7 @@ class Model:
             device = self.tensors[0].device.index if self.tensors and self.tensors[0].is_cuda else 0
         descs, self._keep = _tensor_descs(self.tensors, names)
         self._flush_dir = flush_dir.encode() if flush_dir else None
-        cfg = viper_config(tier, fanout, mode, chunk_bytes, align, device, None, flags, self._flush_dir)
+        cfg = viper_config(tier, fanout, mode, chunk_bytes, align, device, None, flags, self._flush_dir, install_sms)
         if slot1 is not None:
             s1, k1 = _tensor_descs(slot1, names)
             self._keep += [s1, k1]

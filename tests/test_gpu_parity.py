@@ -423,6 +423,36 @@ def test_dram_tier_many_pieces(mode, monkeypatch):
         close_all(prod, cons)
 
 
+@pytest.mark.parametrize("install_sms,cflags,tier", [(1, 0, V.TIER_GPU), (3, V.FLAG_NO_TMA, V.TIER_GPU),
+                                                    (2, 0, V.TIER_DRAM), (500, V.FLAG_NO_TMA, V.TIER_GPU)])
+def test_install_sms_cap(install_sms, cflags, tier):
+    """viper_config.install_sms: ASYNC installs on a capped number of SMs (TMA
+    and register kernels, GPU and DRAM tiers; a cap above the SM count = all)
+    stay byte-exact at ResNet-50 size, where the capped grid runs many rounds
+    of work-counter claims per warp."""
+    specs = synth.model_specs("resnet50")
+    seed = synth.SEEDS["resnet50"]
+    prod_t, cons_t = G.alloc_model(specs), G.alloc_model(specs)
+    name = uname()
+    cons = V.Model(name, V.CONSUMER, cons_t, tier=tier, flags=cflags, install_sms=install_sms)
+    prod = V.Model(name, V.PRODUCER, prod_t, tier=tier, mode=V.ASYNC)
+    try:
+        for v in (1, 2, 3):
+            G.fill_model(prod_t, specs, seed, v)
+            prod.publish(v)
+            cons.wait_installed(v, timeout_us=20_000_000)
+            view = cons.acquire_latest()
+            assert view.version == v
+            assert all(torch.equal(g.view(torch.uint8), p.view(torch.uint8))
+                       for g, p in zip(view.tensors(cons_t), prod_t))
+            cons.release(view)
+        assert cons.stats()["failures"] == 0
+    finally:
+        close_all(prod, [cons])
+    with pytest.raises(V.ViperError):
+        V.Model(uname(), V.CONSUMER, cons_t, install_sms=-1)
+
+
 def test_teardown_races_in_process():
     """Unregistering a producer while its consumers' update threads install
     (ASYNC), and consumers while publishes run, never crashes or hangs."""
