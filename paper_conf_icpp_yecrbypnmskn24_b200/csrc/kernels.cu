@@ -40,6 +40,9 @@ namespace {
 #ifndef VP_FUSED_BLOCKS
 #define VP_FUSED_BLOCKS 2
 #endif
+#ifndef VP_FUSED_READBACK
+#define VP_FUSED_READBACK 1
+#endif
 #ifndef VP_DYNAMIC
 #define VP_DYNAMIC 1  // A/B: profiles/r01/ktime_dynamic_ab.log
 #endif
@@ -228,11 +231,13 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
                 acc += cks_vec(r[u], g0 + 4u * i);
             }
         }
+#if VP_FUSED_READBACK
 #pragma unroll
         for (int u = 0; u < U; u++) {  // read back what this lane stored
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) r[u] = ld_cg(snap + (size_t)i * 16);
         }
+#endif
 #pragma unroll
         for (int k = 0; k < kMaxFused; k++) {
             if (k >= (int)ncons) break;
