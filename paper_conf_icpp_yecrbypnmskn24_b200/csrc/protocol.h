@@ -1,6 +1,7 @@
 // protocol.h -- the host-side version protocol (SURVEY s8(a) a3/a7/a8,
 // DESIGN.md s7), free of CUDA so that it is exercised by CPU multi-process
-// tests (selftest.cpp) exactly as the engine uses it.
+// tests (selftest.cpp) and a ThreadSanitizer build (tests/tsan_protocol.cpp)
+// exactly as the engine uses it.
 //
 //   producer slot reuse  pub_state <- newer; fence; scan pins   (wait_unpinned)
 //   consumer snapshot pin pin <- v; fence; re-read pub_state     (pin_latest)
@@ -48,6 +49,51 @@ inline bool wait_unpinned(Ctrl *ctrl, uint64_t old_v, int64_t timeout_ns, int *w
         }
     }
     return true;
+}
+
+// Consumer: pin the latest published snapshot (v, slot b).  The Dekker pair of
+// wait_unpinned: pin <- v; re-read pub_state; undo if it moved.
+inline bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
+    for (;;) {
+        const uint64_t ps = ctrl->pub_state.load();
+        if (ps == 0) return false;
+        r->pin.store(ps >> 1);
+        if (ctrl->pub_state.load() == ps) {
+            *v = ps >> 1;
+            *b = (int)(ps & 1);
+            return true;
+        }
+        r->pin.store(0);
+    }
+}
+
+// Multi-producer: the version every producer published (all pub_m equal).
+inline bool all_published(Ctrl *ctrl, int M, uint64_t *word) {
+    const uint64_t w0 = ctrl->pub_m[0].load();
+    for (int j = 1; j < M; j++)
+        if (ctrl->pub_m[j].load() != w0) return false;
+    *word = w0;
+    return w0 != 0;
+}
+
+// Multi-producer pin: v once every producer published it, re-validated after the pin.
+inline bool pin_latest_m(Ctrl *ctrl, ConsRec *r, int M, uint64_t *v, int *b) {
+    for (int tries = 0; tries < 1000; tries++) {
+        uint64_t w;
+        if (!all_published(ctrl, M, &w)) {
+            sched_yield();
+            continue;
+        }
+        r->pin.store(w >> 1);
+        uint64_t w2;
+        if (all_published(ctrl, M, &w2) && w2 == w) {
+            *v = w >> 1;
+            *b = (int)(w & 1);
+            return true;
+        }
+        r->pin.store(0);
+    }
+    return false;
 }
 
 // Writer: the alternative copy is written only once no reader pins it.

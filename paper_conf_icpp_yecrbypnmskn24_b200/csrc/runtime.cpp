@@ -282,48 +282,6 @@ void fire_callback(viper_model *c, uint64_t v, viper_status st) {
 // Pin the latest published snapshot (Dekker pair with the producer's
 // pub_state store -> pin scan).  Returns false when
 // nothing is published.
-// Multi-producer: the version every producer published (all pub_m equal).
-static bool all_published(Ctrl *ctrl, int M, uint64_t *word) {
-    const uint64_t w0 = ctrl->pub_m[0].load();
-    for (int j = 1; j < M; j++)
-        if (ctrl->pub_m[j].load() != w0) return false;
-    *word = w0;
-    return w0 != 0;
-}
-
-bool pin_latest_m(Ctrl *ctrl, ConsRec *r, int M, uint64_t *v, int *b) {
-    for (int tries = 0; tries < 1000; tries++) {
-        uint64_t w;
-        if (!all_published(ctrl, M, &w)) {
-            sched_yield();
-            continue;
-        }
-        r->pin.store(w >> 1);
-        uint64_t w2;
-        if (all_published(ctrl, M, &w2) && w2 == w) {
-            *v = w >> 1;
-            *b = (int)(w & 1);
-            return true;
-        }
-        r->pin.store(0);
-    }
-    return false;
-}
-
-bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b) {
-    for (;;) {
-        const uint64_t ps = ctrl->pub_state.load();
-        if (ps == 0) return false;
-        r->pin.store(ps >> 1);
-        if (ctrl->pub_state.load() == ps) {
-            *v = ps >> 1;
-            *b = (int)(ps & 1);
-            return true;
-        }
-        r->pin.store(0);
-    }
-}
-
 // Host half of an install of snapshot slot b (version v) of producer p into
 // the inactive slot of consumer c: wait until no reader pins the target (a7)
 // and build the kernel arguments.  Caller holds c->install_mu.

@@ -227,7 +227,6 @@ viper_status build_manifest(Manifest &m, const viper_tensor *t, int32_t n, uint6
 viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, Item **d_out, uint32_t share_n,
                           uint32_t share_me, uint32_t *count);
 std::atomic<uint64_t> &pub_word(viper_model *p);
-bool pin_latest(Ctrl *ctrl, ConsRec *r, uint64_t *v, int *b);
 viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, int b, PreparedInstall *pi);
 viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, cudaStream_t st, bool wait_ready,
                              bool pdl);
