@@ -494,6 +494,70 @@ N_CONFIG = {2: "resnet50", 4: "vit_b16", 8: "gpt2_xl"}  # BASELINE.json configs[
 CONFIG_INDEX = {"ptychonn": 0, "resnet50": 1, "vit_b16": 2, "gpt2_xl": 3, "llama3_8b": 4}
 
 
+def xproc_e2e(V, G, synth, name, rank, world, dev, group, fanout, flush_buf, steps, warmup):
+    """The N > 1 update end to end through the public API with HOST buffers
+    (the N = 1 run_e2e across processes).  Rank 0's parameters live in one flat
+    device buffer; each step copies the step's weights from a pinned host
+    buffer (one H2D of S bytes), publishes SYNC (returns after every consumer
+    swapped), and reads the chunk-seal digest back (D2H).  Rank 0's host clock
+    around the three; the consumers only take part in the publishes."""
+    import torch
+    import torch.distributed as dist
+    specs = synth.model_specs(name)
+    offs, off = [], 0
+    for s_ in specs:
+        offs.append(off)
+        off = (off + synth.nbytes_of(s_) + 255) // 256 * 256
+    dt = {synth.F32: torch.float32, synth.BF16: torch.bfloat16, synth.F16: torch.float16}
+    flat = torch.empty(max(off, 256), dtype=torch.uint8, device="cuda")
+    tensors = [flat[o:o + synth.nbytes_of(s_)].view(dt.get(s_[1], torch.uint8)).view(s_[2])
+               for o, s_ in zip(offs, specs)]
+    host, digest = [], None
+    if rank == 0:
+        for i in range(2):  # two host versions of the whole flat buffer, alternated
+            G.fill_model(tensors, specs, synth.SEEDS[name], 1000 + i)
+            hb = G.PinnedBuffer(flat.numel())
+            hb.view()[:] = flat.cpu().numpy()
+            host.append(hb)
+    bs = V.Bootstrap(rank, world, producer_rank=0, group=group)
+    m = V.Model(f"bench-x-e2e-{name}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors, fanout=fanout,
+                device=dev, bootstrap=bs)
+    times, ok, nchunks = [], True, 0
+    try:
+        if rank == 0:
+            _, _, nchunks = m.debug_buffers()
+            digest = G.PinnedBuffer(16 * nchunks)
+        st = torch.cuda.current_stream()
+        for i in range(warmup + steps):
+            G.l2_flush(flush_buf, stream=st)
+            torch.cuda.synchronize()
+            dist.barrier(group=group)
+            if rank == 0:
+                t0 = time.perf_counter()
+                host[i % 2].to_device(flat, stream=st)
+                m.publish(i + 1, stream=st)
+                _, seals_ptr, _ = m.debug_buffers()
+                digest.from_device_ptr(seals_ptr, 16 * nchunks, stream=st)
+                st.synchronize()
+                if i >= warmup:
+                    times.append((time.perf_counter() - t0) * 1e3)
+            dist.barrier(group=group)
+        if rank == 0:
+            d = digest.view().view("<u8").reshape(nchunks, 2)
+            ok = bool((d[:, 0] == warmup + steps).all())
+    finally:
+        if rank != 0:  # consumers first, as in xproc_arm
+            m.close()
+        dist.barrier(group=group)
+        if rank == 0:
+            m.close()
+        for hb in host:
+            hb.close()
+        if digest is not None:
+            digest.close()
+    return {"ms": statistics.mean(times) if times else 0.0, "h2d": flat.numel(), "d2h": 16 * nchunks, "ok": ok}
+
+
 def xproc_arm(args):
     """N > 1: one process per GPU.  Rank 0 is the producer, ranks 1..N-1 the
     consumers (1 -> N-1 fan-out over NVLink: direct for one consumer,
@@ -573,9 +637,12 @@ def xproc_arm(args):
         e1.synchronize()
         if i >= args.warmup:
             nccl_ms.append(e0.elapsed_time(e1))
+    del buf
+    e2e = xproc_e2e(V, G, synth, name, rank, world, dev, gloo, fanout, flush, args.steps, args.warmup)
     t = torch.tensor([statistics.mean(lat[args.warmup:]) if rank == 0 else 0.0,
                       statistics.median(inst[args.warmup:]) if rank else 0.0,
-                      statistics.mean(nccl_ms), float(1 - ok)], dtype=torch.float64)
+                      statistics.mean(nccl_ms), float(1 - ok), e2e["ms"], float(1 - e2e["ok"])],
+                     dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
     if rank != 0:
         m.close()
@@ -605,7 +672,10 @@ def xproc_arm(args):
             "parity_ok": bool(float(t[3]) == 0.0),
             "gpu_launches": 3 * args.steps,
             "clocks": clk.summary(),
-            "e2e": None,
+            "e2e": {"value": round(float(t[4]), 6), "unit": "ms", "h2d_bytes_per_step": e2e["h2d"],
+                    "d2h_bytes_per_step": e2e["d2h"], "digest_ok": bool(float(t[5]) == 0.0),
+                    "how": "rank 0: pinned host -> device copy of the step's weights, SYNC publish (returns "
+                           "after every consumer swapped), D2H of the chunk-seal digest; host clock"},
         }
         print(json.dumps(out), flush=True)
     dist.barrier(group=gloo)

@@ -120,7 +120,15 @@ enum { VIPER_FLAG_TIMING = 2,   /* record CUDA events around the pack / install 
                                    applies: packs no install is PDL-chained to
                                    (ASYNC, DRAM tier, cross-process) and direct
                                    installs of a completed snapshot               */
-       VIPER_FLAG_NO_TMA = 16 }; /* never auto-select the TMA kernels             */
+       VIPER_FLAG_NO_TMA = 16,  /* never auto-select the TMA kernels (the fused
+                                   SYNC kernel streams through registers)         */
+       VIPER_FLAG_FUSED_TMA = 32 }; /* producer: the fused SYNC kernel moves every
+                                   16-B-aligned item with TMA bulk copies (one
+                                   shared-memory stage stored into the snapshot
+                                   and every consumer slot) and verifies the
+                                   installed slot bytes by reading them back.
+                                   Never auto-selected: it measured slower than
+                                   the register fused kernel       */
 
 typedef struct {
     int32_t tier;            /* VIPER_TIER_*                       (default GPU)    */

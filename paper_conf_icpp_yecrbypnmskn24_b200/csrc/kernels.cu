@@ -783,7 +783,241 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
     install_finish(a, bad);
 }
 
+// ---------------------------------------------------------------------------
+// publish_fused, TMA bulk-copy variant (SYNC in-process).  Per warp, a ring of
+// kFtStages shared-memory stages of kFtStage bytes (>= the default 8 KiB item
+// cap, so an item is one piece).  Lane 0 brings each item's piece in with
+// cp.async.bulk (global -> shared, mbarrier complete_tx); all lanes checksum
+// it from shared memory (the item seal); lane 0 then issues bulk stores of
+// the SAME stage into the snapshot and into every consumer's inactive slot
+// (one bulk group per piece).  Install verification (R21'): once an
+// item's bulk group has completed -- checked one item later, so the wait
+// overlaps the next item's stream -- the warp reads the installed slot bytes
+// back (L2 hits) and recomputes their checksum against the seal.  Items that
+// are not 16-B aligned (or have a <16-B tail) take the register path
+// (copy_item_fused) inline.  Static strided items.
+#ifndef VP_FT_WARPS
+#define VP_FT_WARPS 4
+#endif
+#ifndef VP_FT_STAGES
+#define VP_FT_STAGES 3
+#endif
+#ifndef VP_FT_STAGE
+#define VP_FT_STAGE 8192
+#endif
+#ifndef VP_FT_READBACK
+#define VP_FT_READBACK 1
+#endif
+constexpr int kFtWarps = VP_FT_WARPS;
+constexpr int kFtStages = VP_FT_STAGES;
+constexpr uint32_t kFtStage = VP_FT_STAGE;
+
+__device__ __forceinline__ void bulk_s2g_nc(void *gmem, const void *smem, uint32_t bytes) {  // no commit
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gmem), "r"(smem_u32(smem)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+// 16-B-aligned TMA body of fused item w (0: the whole item takes the register path)
+__device__ __forceinline__ uint32_t fused_tma_body(const FusedArgs &a, const Item &it, uint32_t w) {
+    uint64_t m = it.ptr | it.packed_off | it.nbytes;
+#pragma unroll
+    for (int k = 0; k < kMaxFused; k++)
+        if (k < (int)a.ncons) m |= a.cons[k].items[w].ptr;
+    return (m & 15u) ? 0u : it.nbytes;
+}
+
+// Read consumer k's installed copy of item w back and checksum it (after the
+// item's bulk stores completed).  Returns the bit mask of consumers whose copy
+// does not match `sealed`.  Fault injection flips the first word first.
+__device__ __forceinline__ uint32_t fused_verify_slots(const FusedArgs &a, uint32_t w, uint64_t sealed,
+                                                       uint32_t lane) {
+    const Item it = a.items[w];
+    const uint32_t nvec = it.nbytes >> 4;
+    const uint32_t g0 = (uint32_t)(it.packed_off >> 2);
+    uint32_t bad = 0;
+#pragma unroll
+    for (int k = 0; k < kMaxFused; k++) {
+        if (k >= (int)a.ncons) break;
+        const uint8_t *dst = (const uint8_t *)a.cons[k].items[w].ptr;
+        if (w == a.cons[k].fault_item) {
+            if (lane == 0) *(volatile uint32_t *)dst ^= 0x10u;
+            __syncwarp();
+        }
+        uint64_t c = 0;
+        for (uint32_t base = 0; base < nvec; base += 32 * kFusedUnroll) {
+            uint4 r[kFusedUnroll];
+#pragma unroll
+            for (int u = 0; u < kFusedUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) r[u] = ld_cg(dst + (size_t)i * 16);
+            }
+#pragma unroll
+            for (int u = 0; u < kFusedUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) c += cks_vec(r[u], g0 + 4u * i);
+            }
+        }
+        if (warp_sum(c) + a.version * kVerMix != sealed) bad |= 1u << k;
+    }
+    return bad;
+}
+
+__global__ void __launch_bounds__(kFtWarps * 32, 2) publish_fused_tma_kernel(const FusedArgs a) {
+    extern __shared__ __align__(128) uint8_t tma_smem[];
+    const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    uint8_t *stage = tma_smem + wib * (kFtStages * kFtStage);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(tma_smem + kFtWarps * kFtStages * kFtStage) + wib * kFtStages;
+    if (lane == 0) {
+        for (int s = 0; s < kFtStages; s++) mbar_init(bar + s);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    const uint32_t nwarps = gridDim.x * kFtWarps;
+    const uint32_t w0 = blockIdx.x * kFtWarps + wib;
+    TmaCursor ld{w0, 0};
+    auto next_piece = [&](TmaCursor &c, Item &it, uint32_t &bytes) -> bool {
+        while (c.w < a.nitems) {
+            it = a.items[c.w];
+            const uint32_t body = fused_tma_body(a, it, c.w);
+            if (c.off < body) {
+                bytes = min(kFtStage, body - c.off);
+                return true;
+            }
+            c.w += nwarps;
+            c.off = 0;
+        }
+        return false;
+    };
+    for (int s = 0; s < kFtStages; s++) {  // prologue: fill the ring
+        Item it;
+        uint32_t bytes;
+        if (!next_piece(ld, it, bytes)) break;
+        if (lane == 0) {
+            mbar_expect_tx(bar + s, bytes);
+            bulk_g2s(stage + s * kFtStage, (const uint8_t *)it.ptr + ld.off, bytes, bar + s);
+        }
+        ld.off += bytes;
+    }
+    uint32_t consumed = 0, phase_bits = 0, bad = 0;
+    uint32_t pw = 0xffffffffu;  // previous TMA item: verified once its bulk group completed
+    uint64_t psealed = 0;
+    for (uint32_t w = w0; w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        const uint32_t body = fused_tma_body(a, it, w);
+        if (body == 0) {  // register path, verified inline (copy_item_fused's read-back)
+            uint64_t cptr[kMaxFused];
+            uint32_t inject = 0;
+#pragma unroll
+            for (int k = 0; k < kMaxFused; k++) {
+                cptr[k] = k < (int)a.ncons ? a.cons[k].items[w].ptr : 0;
+                if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
+            }
+            uint64_t got[kMaxFused] = {0, 0, 0, 0};
+            const uint64_t sealed =
+                warp_sum(copy_item_fused<kFusedUnroll>((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
+                                                       a.ncons, it.nbytes, it.packed_off, lane, inject, got)) +
+                a.version * kVerMix;
+            if (lane == 0) {
+                a.iseal[w].mixed = sealed;
+                a.iseal[w].version = a.version;
+            }
+#pragma unroll
+            for (int k = 0; k < kMaxFused; k++) {
+                if (k >= (int)a.ncons) break;
+                if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
+            }
+            continue;
+        }
+        uint64_t acc = 0;
+        uint32_t npieces = 0;
+        for (uint32_t off = 0; off < body; off += kFtStage) {
+            const uint32_t bytes = min(kFtStage, body - off);
+            const int s = consumed % kFtStages;
+            mbar_wait(bar + s, (phase_bits >> s) & 1u);
+            phase_bits ^= 1u << s;
+            const uint8_t *buf = stage + s * kFtStage;
+            const uint32_t g0 = (uint32_t)((it.packed_off + off) >> 2);
+            for (uint32_t i = lane; i < bytes / 16; i += 32)
+                acc += cks_vec(*reinterpret_cast<const uint4 *>(buf + i * 16), g0 + 4u * i);
+            __syncwarp();
+            if (lane == 0) {
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                bulk_s2g_nc(a.packed + it.packed_off + off, buf, bytes);
+                for (uint32_t k = 0; k < a.ncons; k++) bulk_s2g_nc((uint8_t *)a.cons[k].items[w].ptr + off, buf, bytes);
+                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            }
+            consumed++;
+            npieces++;
+            Item nit;
+            uint32_t nbytes;
+            if (next_piece(ld, nit, nbytes)) {  // refill this stage once the stores have read it
+                if (lane == 0) {
+                    bulk_wait_read<0>();
+                    mbar_expect_tx(bar + s, nbytes);
+                    bulk_g2s(stage + s * kFtStage, (const uint8_t *)nit.ptr + ld.off, nbytes, bar + s);
+                }
+                ld.off += nbytes;
+            }
+        }
+        const uint64_t sealed = warp_sum(acc) + a.version * kVerMix;
+        if (lane == 0) {  // no concurrent reader in this path: a plain store (grid end publishes it)
+            a.iseal[w].mixed = sealed;
+            a.iseal[w].version = a.version;
+        }
+        if (VP_FT_READBACK && pw != 0xffffffffu) {
+            // the previous item's group completed once at most this item's
+            // `npieces` groups are still pending
+            if (lane == 0) {
+                if (npieces == 1) asm volatile("cp.async.bulk.wait_group 1;" ::: "memory");
+                else asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+                asm volatile("fence.proxy.async.global;" ::: "memory");
+            }
+            __syncwarp();
+            bad |= fused_verify_slots(a, pw, psealed, lane);
+        }
+        pw = w;
+        psealed = sealed;
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;\n\tfence.proxy.async.global;" ::: "memory");
+    __syncwarp();
+    if (VP_FT_READBACK && pw != 0xffffffffu) bad |= fused_verify_slots(a, pw, psealed, lane);
+    if (lane == 0 && bad) report_err(a.flags, bad);
+    __syncthreads();
+    uint32_t e;
+    if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
+        for (uint32_t k = 0; k < a.ncons; k++) {
+            const FusedCons &c = a.cons[k];
+            const int32_t st = (e >> k) & 1u ? -5 : 0;
+            if (c.status_h) *c.status_h = st;
+            if (st == 0 && c.state_h) *c.state_h = (a.version << 1) | (uint64_t)c.target;  // the swap
+            if (c.pin_h) *c.pin_h = 0;
+        }
+    }
+}
+
 }  // namespace
+
+FusedLaunch fused_tma_launch(uint32_t nitems, int device) {
+    static int sms = 0;
+    static size_t smem = 0;
+    FusedLaunch l{};
+    l.func = (const void *)publish_fused_tma_kernel;
+    l.smem = kFtWarps * kFtStages * kFtStage + kFtWarps * kFtStages * sizeof(uint64_t);
+    if (sms == 0) {
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) sms = 148;
+    }
+    if (smem != l.smem) {
+        l.err = cudaFuncSetAttribute(publish_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)l.smem);
+        if (l.err != cudaSuccess) return l;
+        smem = l.smem;
+    }
+    const uint32_t want = (nitems + kFtWarps - 1) / kFtWarps;
+    const uint32_t cap = (uint32_t)sms * 2;
+    l.grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+    l.block = kFtWarps * 32;
+    return l;
+}
 
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
     static int sms = 0;

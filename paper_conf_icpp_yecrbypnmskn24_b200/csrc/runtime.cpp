@@ -520,13 +520,29 @@ static const bool g_trace_on = getenv("VIPER_TRACE") != nullptr;  // tools/trace
 // (profiles/r01/launchcal.log).  VIPER_NO_GRAPH=1 launches directly.
 static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStream_t st) {
     static const bool no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));
+    static const int tma_env = getenv("VIPER_FUSED_TMA") ? atoi(getenv("VIPER_FUSED_TMA")) : -1;
+    const int32_t fl = p->cfg.flags;
+    const bool tma = tma_env >= 0                  ? tma_env != 0
+                     : (fl & VIPER_FLAG_FUSED_TMA) ? true
+                     : (fl & VIPER_FLAG_NO_TMA)    ? false
+                                                   : kFusedTmaDefault && p->man.s_packed <= kFusedTmaMaxBytes;
     const Geometry fg = fused_geometry(p->geo);
-    if (no_graph) return launch_fused(f, fg, st);
     void *args[] = {(void *)&f};
     cudaKernelNodeParams kp{};
-    kp.func = (void *)fused_kernel_fn();
-    kp.gridDim = dim3(fg.grid);
-    kp.blockDim = dim3(fg.block);
+    if (tma) {
+        const FusedLaunch l = fused_tma_launch(f.nitems, p->device);
+        if (l.err != cudaSuccess) return l.err;
+        kp.func = (void *)l.func;
+        kp.gridDim = dim3(l.grid);
+        kp.blockDim = dim3(l.block);
+        kp.sharedMemBytes = (unsigned)l.smem;
+        if (no_graph) return cudaLaunchKernel(l.func, kp.gridDim, kp.blockDim, args, l.smem, st);
+    } else {
+        if (no_graph) return launch_fused(f, fg, st);
+        kp.func = (void *)fused_kernel_fn();
+        kp.gridDim = dim3(fg.grid);
+        kp.blockDim = dim3(fg.block);
+    }
     kp.kernelParams = args;
     cudaError_t e;
     if (!p->fused_exec) {

@@ -139,6 +139,21 @@ cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
 const void *fused_kernel_fn();  // for the one-node launch graph (runtime.cpp)
+// TMA bulk-copy variant of the fused kernel: function, geometry and dynamic
+// shared memory for the launch graph (err != cudaSuccess: not launchable)
+struct FusedLaunch {
+    const void *func;
+    int grid, block;
+    size_t smem;
+    cudaError_t err;
+};
+FusedLaunch fused_tma_launch(uint32_t nitems, int device);
+#ifndef VP_FUSED_TMA_DEFAULT
+#define VP_FUSED_TMA_DEFAULT 0
+#endif
+// SYNC in-process publishes use the TMA fused kernel (VIPER_FUSED_TMA=0/1 overrides)
+constexpr bool kFusedTmaDefault = VP_FUSED_TMA_DEFAULT != 0;
+constexpr uint64_t kFusedTmaMaxBytes = 1ull << 30;  // auto-selection limit (packed bytes)
 // pdl: the install directly follows the pack on `st` (programmatic dependent launch)
 cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl);
 

@@ -23,6 +23,7 @@ FLAG_TIMING = 2
 FLAG_NO_FUSE = 4
 FLAG_TMA = 8
 FLAG_NO_TMA = 16
+FLAG_FUSED_TMA = 32
 SCHED_FIXED, SCHED_GREEDY = 0, 1
 
 

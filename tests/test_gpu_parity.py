@@ -79,6 +79,7 @@ def close_all(prod, cons):
 
 # ------------------------------------------------------------------ C1 (BJ configs[0])
 @pytest.mark.parametrize("tier,mode,flags", [(V.TIER_GPU, V.SYNC, 0), (V.TIER_GPU, V.SYNC, V.FLAG_NO_FUSE),
+                                              (V.TIER_GPU, V.SYNC, V.FLAG_FUSED_TMA),
                                               (V.TIER_GPU, V.SYNC, V.FLAG_TMA), (V.TIER_GPU, V.ASYNC, V.FLAG_TMA),
                                               (V.TIER_GPU, V.ASYNC, 0), (V.TIER_DRAM, V.SYNC, 0),
                                               (V.TIER_DRAM, V.ASYNC, 0)])
@@ -120,7 +121,7 @@ def test_ragged_tensor_lists_many_chunks(seed):
         specs.append((f"t{i}", dt, (ne,)))
     chunk = int(rng.choice([256, 4096, 65536]))
     align = int(rng.choice([16, 256]))
-    flags = [0, V.FLAG_NO_FUSE, V.FLAG_TMA][seed % 3]
+    flags = [0, V.FLAG_NO_FUSE, V.FLAG_TMA, V.FLAG_FUSED_TMA][seed % 4]
     ncons = 3 if seed < 4 else 6   # > kMaxFused local consumers -> separate kernels
     prod, prod_t, cons, cons_t = make_pair(specs, seed, ncons=ncons, chunk_bytes=chunk, align=align, flags=flags)
     try:
@@ -179,7 +180,7 @@ def test_empty_model():
 
 
 # ---------------------------------------------------------------- protocol on device
-@pytest.mark.parametrize("flags", [0, V.FLAG_NO_FUSE])
+@pytest.mark.parametrize("flags", [0, V.FLAG_NO_FUSE, V.FLAG_FUSED_TMA, V.FLAG_NO_TMA])
 def test_fault_injection_keeps_old_version(flags):
     specs = synth.model_specs("ptychonn")
     seed = 11
@@ -353,6 +354,9 @@ def test_no_torn_reads_under_async_publishes():
 @pytest.mark.parametrize("name,flags,tier", [("resnet50", 0, V.TIER_GPU), ("vit_b16", 0, V.TIER_GPU),
                                              ("gpt2_xl", 0, V.TIER_GPU), ("llama3_8b", 0, V.TIER_GPU),
                                              ("gpt2_xl", V.FLAG_TMA, V.TIER_GPU), ("resnet50", 0, V.TIER_DRAM),
+                                             ("resnet50", V.FLAG_FUSED_TMA, V.TIER_GPU),
+                                             ("resnet50", V.FLAG_NO_TMA, V.TIER_GPU),
+                                             ("gpt2_xl", V.FLAG_FUSED_TMA, V.TIER_GPU),
                                              ("gpt2_xl", 0, V.TIER_DRAM),
                                              # register pack + PDL register install: > one round of items per
                                              # warp, so both work counters hand out items (kernels.cu WorkQueue)
@@ -546,7 +550,7 @@ def test_randomized_configurations(seed):
         specs.append((f"t{i}", dt, (ne,)))
     mode = int(rng.choice([V.SYNC, V.ASYNC]))
     tier = int(rng.choice([V.TIER_GPU, V.TIER_DRAM]))
-    flags = int(rng.choice([0, V.FLAG_NO_FUSE, V.FLAG_TMA, V.FLAG_NO_TMA]))
+    flags = int(rng.choice([0, V.FLAG_NO_FUSE, V.FLAG_TMA, V.FLAG_NO_TMA, V.FLAG_FUSED_TMA]))
     chunk = int(rng.choice([4096, 65536, 2 << 20]))
     align = int(rng.choice([16, 256]))
     ncons = int(rng.integers(1, 6))

@@ -24,7 +24,8 @@ pt, ct = G.alloc_model(specs), G.alloc_model(specs)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 S = synth.model_bytes(a.config)
 res = {}
-for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE | V.FLAG_NO_TMA), ("tma", V.FLAG_TMA)):
+for label, flags in (("fused", V.FLAG_NO_TMA), ("fused_tma", V.FLAG_FUSED_TMA), ("sep", V.FLAG_NO_FUSE | V.FLAG_NO_TMA),
+                     ("tma", V.FLAG_TMA)):
     cflags = {"sep": V.FLAG_NO_TMA, "tma": V.FLAG_TMA}.get(label, 0)
     c = V.Model("kt" + label, V.CONSUMER, ct, flags=V.FLAG_TIMING | cflags)
     p = V.Model("kt" + label, V.PRODUCER, pt, flags=V.FLAG_TIMING | flags)
@@ -44,8 +45,8 @@ for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE | V.FLAG_NO_TMA), ("tm
             ins.append(c.stats()["t_install_dev_us"])
     c.close()
     p.close()
-    if label == "fused":
-        res["fused"] = statistics.median(fu)
+    if label in ("fused", "fused_tma"):
+        res[label] = statistics.median(fu)
     elif label == "sep":
         res["pack"], res["install"] = statistics.median(pk), statistics.median(ins)
     else:
@@ -53,6 +54,7 @@ for label, flags in (("fused", 0), ("sep", V.FLAG_NO_FUSE | V.FLAG_NO_TMA), ("tm
         res["install_tma"] = statistics.median(ins)
 lib = os.path.basename(os.environ.get("VIPER_LIB_PATH", "libviper.so"))
 print(f"{lib:28s} {a.config:9s} fused {res['fused']:9.2f} us ({3*S/res['fused']/1e3/6550.4:.3f})  "
+      f"fused_tma {res['fused_tma']:9.2f} us ({3*S/res['fused_tma']/1e3/6550.4:.3f})  "
       f"pack {res['pack']:9.2f} us ({2*S/res['pack']/1e3/6550.4:.3f})  "
       f"install {res['install']:9.2f} us ({2*S/res['install']/1e3/6550.4:.3f})  "
       f"pack_tma {res['tma']:9.2f} us ({2*S/res['tma']/1e3/6550.4:.3f})  "
