@@ -43,6 +43,9 @@ namespace {
 #ifndef VP_FUSED_READBACK
 #define VP_FUSED_READBACK 1
 #endif
+#ifndef VP_WARP_PROF
+#define VP_WARP_PROF 0  // tools/warp_prof.py builds a side variant with per-warp timestamps
+#endif
 #ifndef VP_DYNAMIC
 #define VP_DYNAMIC 1  // A/B: profiles/r01/ktime_dynamic_ab.log
 #endif
@@ -480,11 +483,27 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
 // exactly the snapshot bytes it stored (same thread, so ordered) with L2
 // loads, installs them and recomputes the item checksum; the seal check is
 // against the value just sealed.  No cross-warp dependency inside the grid.
+#if VP_WARP_PROF
+// tools/warp_prof.py (profiling builds only): per warp {start, end, items, bytes}
+__device__ unsigned long long g_warp_prof[8192 * 4];
+__device__ unsigned long long g_prof_end;  // the last block, after the swap
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#endif
+
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fused_kernel(const FusedArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+#if VP_WARP_PROF
+    const uint32_t gw = w;
+    const unsigned long long prof_t0 = gtimer();
+    unsigned long long prof_items = 0, prof_bytes = 0;
+#endif
     WorkQueue q(reinterpret_cast<unsigned int *>(a.flags + 1), 0, nwarps, a.nitems);  // reset by the last block
     if (w < a.nitems) q.claim(lane);
     while (w < a.nitems) {
@@ -509,9 +528,21 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
             if (k >= (int)a.ncons) break;
             if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
         }
+#if VP_WARP_PROF
+        prof_items++;
+        prof_bytes += it.nbytes;
+#endif
         w = q.next(w, lane);
         if (w < a.nitems) q.claim(lane);
     }
+#if VP_WARP_PROF
+    if (lane == 0 && gw < 8192) {
+        g_warp_prof[gw * 4 + 0] = prof_t0;
+        g_warp_prof[gw * 4 + 1] = gtimer();
+        g_warp_prof[gw * 4 + 2] = prof_items;
+        g_warp_prof[gw * 4 + 3] = prof_bytes;
+    }
+#endif
     if (lane == 0 && bad) report_err(a.flags, bad);
     __syncthreads();
     uint32_t e;
@@ -524,6 +555,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
             if (st == 0 && c.state_h) *c.state_h = (a.version << 1) | (uint64_t)c.target;  // the swap
             if (c.pin_h) *c.pin_h = 0;
         }
+#if VP_WARP_PROF
+        g_prof_end = gtimer();
+#endif
     }
 }
 
@@ -997,6 +1031,14 @@ __global__ void __launch_bounds__(kFtWarps * 32, 2) publish_fused_tma_kernel(con
 }
 
 }  // namespace
+
+#if VP_WARP_PROF
+extern "C" int vp_debug_warp_prof(unsigned long long *out, int nwarps) {
+    cudaError_t e = cudaMemcpyFromSymbol(out, g_warp_prof, sizeof(unsigned long long) * 4 * (size_t)nwarps);
+    if (e == cudaSuccess) e = cudaMemcpyFromSymbol(out + 4 * (size_t)nwarps, g_prof_end, sizeof(unsigned long long));
+    return (int)e;
+}
+#endif
 
 FusedLaunch fused_tma_launch(uint32_t nitems, int device) {
     static int sms = 0;
