@@ -21,6 +21,8 @@
 // side stream.
 #include "vp_internal.h"
 
+#include <atomic>
+
 namespace vp {
 
 namespace {
@@ -1040,38 +1042,55 @@ extern "C" int vp_debug_warp_prof(unsigned long long *out, int nwarps) {
 }
 #endif
 
+// Per-device launch facts, cached once per (kernel, device): the SM count and
+// the dynamic shared-memory opt-in (cudaFuncSetAttribute applies to the
+// current device only).  Lock-free; a race just repeats idempotent calls.
+constexpr int kMaxDevices = 64;
+
+static int sm_count(int device) {
+    static std::atomic<int> cache[kMaxDevices];
+    const int d = device >= 0 && device < kMaxDevices ? device : 0;
+    int n = cache[d].load(std::memory_order_relaxed);
+    if (n > 0) return n;
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || n <= 0) n = 148;
+    cache[d].store(n, std::memory_order_relaxed);
+    return n;
+}
+
+template <typename Kernel>
+static cudaError_t opt_in_smem(Kernel kernel, size_t smem, int device, std::atomic<uint64_t> &done) {
+    const uint64_t bit = 1ull << (device >= 0 && device < kMaxDevices ? device : 0);
+    if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+    const cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+    return e;  // not cached on failure: the next launch retries and reports again
+}
+
+static int grid_for(uint32_t nitems, int warps_per_block, int sms, int blocks_per_sm) {
+    const uint32_t want = (nitems + warps_per_block - 1) / warps_per_block;
+    const uint32_t cap = (uint32_t)sms * blocks_per_sm;
+    return (int)(want < 1 ? 1 : (want > cap ? cap : want));
+}
+
+constexpr size_t kTmaSmem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
+
 FusedLaunch fused_tma_launch(uint32_t nitems, int device) {
-    static int sms = 0;
-    static size_t smem = 0;
+    static std::atomic<uint64_t> opted{0};
     FusedLaunch l{};
     l.func = (const void *)publish_fused_tma_kernel;
     l.smem = kFtWarps * kFtStages * kFtStage + kFtWarps * kFtStages * sizeof(uint64_t);
-    if (sms == 0) {
-        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) sms = 148;
-    }
-    if (smem != l.smem) {
-        l.err = cudaFuncSetAttribute(publish_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)l.smem);
-        if (l.err != cudaSuccess) return l;
-        smem = l.smem;
-    }
-    const uint32_t want = (nitems + kFtWarps - 1) / kFtWarps;
-    const uint32_t cap = (uint32_t)sms * 2;
-    l.grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+    l.err = opt_in_smem(publish_fused_tma_kernel, l.smem, device, opted);
+    l.grid = grid_for(nitems, kFtWarps, sm_count(device), 2);
     l.block = kFtWarps * 32;
     return l;
 }
 
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
-    static int sms = 0;
-    if (sms == 0) {
-        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess || sms <= 0) sms = 148;
-    }
+    const int sms = sm_count(device);
     Geometry g;
     g.items = nitems;
     g.block = kWarpsPerBlock * 32;
-    const uint32_t want = (nitems + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    const uint32_t cap = (uint32_t)(max_sms > 0 && max_sms < sms ? max_sms : sms) * kBlocksPerSM;
-    g.grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
+    g.grid = grid_for(nitems, kWarpsPerBlock, max_sms > 0 && max_sms < sms ? max_sms : sms, kBlocksPerSM);
     return g;
 }
 
@@ -1083,30 +1102,19 @@ cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
 
 cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
     if (a.nitems == 0) return cudaSuccess;
-    static int sms = 0;
-    const size_t smem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
-    if (sms == 0) {
-        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) sms = 148;
-        cudaError_t e = cudaFuncSetAttribute(pack_seal_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-    }
-    const uint32_t want = (a.nitems + kTmaWarps - 1) / kTmaWarps;
-    const uint32_t cap = (uint32_t)sms * 2;
-    const int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    pack_seal_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
+    static std::atomic<uint64_t> opted{0};
+    const cudaError_t e = opt_in_smem(pack_seal_tma_kernel, kTmaSmem, device, opted);
+    if (e != cudaSuccess) return e;
+    pack_seal_tma_kernel<<<grid_for(a.nitems, kTmaWarps, sm_count(device), 2), kTmaWarps * 32, kTmaSmem, st>>>(a);
     return cudaGetLastError();
 }
 
 const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
 
-Geometry fused_geometry(const Geometry &g) {
+Geometry fused_geometry(const Geometry &g, int device) {
     // same block shape, up to kFusedBlocks resident blocks per SM
     Geometry f = g;
-    static int sms = 0;
-    if (sms == 0 && (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0) != cudaSuccess || sms <= 0)) sms = 148;
-    const int cap = sms * kFusedBlocks;
-    const int want = (int)((g.items + kWarpsPerBlock - 1) / kWarpsPerBlock);
-    f.grid = want < 1 ? 1 : (want > cap ? cap : want);
+    f.grid = grid_for(g.items, kWarpsPerBlock, sm_count(device), kFusedBlocks);
     return f;
 }
 
@@ -1116,18 +1124,12 @@ cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st)
 }
 
 cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device, int max_sms) {
-    static int sms = 0;
-    const size_t smem = (size_t)kTmaWarps * kTmaStages * kTmaStage + kTmaWarps * kTmaStages * sizeof(uint64_t);
-    if (sms == 0) {
-        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) sms = 148;
-        cudaError_t e =
-            cudaFuncSetAttribute(install_verify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-    }
-    const uint32_t want = (a.nitems + kTmaWarps - 1) / kTmaWarps;
-    const uint32_t cap = (uint32_t)(max_sms > 0 && max_sms < sms ? max_sms : sms) * 2;
-    const int grid = (int)(want < 1 ? 1 : (want > cap ? cap : want));
-    install_verify_tma_kernel<<<grid, kTmaWarps * 32, smem, st>>>(a);
+    static std::atomic<uint64_t> opted{0};
+    const cudaError_t e = opt_in_smem(install_verify_tma_kernel, kTmaSmem, device, opted);
+    if (e != cudaSuccess) return e;
+    const int sms = sm_count(device);
+    const int grid = grid_for(a.nitems, kTmaWarps, max_sms > 0 && max_sms < sms ? max_sms : sms, 2);
+    install_verify_tma_kernel<<<grid, kTmaWarps * 32, kTmaSmem, st>>>(a);
     return cudaGetLastError();
 }
 

@@ -526,7 +526,7 @@ static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStr
                      : (fl & VIPER_FLAG_FUSED_TMA) ? true
                      : (fl & VIPER_FLAG_NO_TMA)    ? false
                                                    : kFusedTmaDefault && p->man.s_packed <= kFusedTmaMaxBytes;
-    const Geometry fg = fused_geometry(p->geo);
+    const Geometry fg = fused_geometry(p->geo, p->device);
     void *args[] = {(void *)&f};
     cudaKernelNodeParams kp{};
     if (tma) {

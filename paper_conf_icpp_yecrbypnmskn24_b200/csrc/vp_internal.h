@@ -128,7 +128,7 @@ struct Geometry {
     int grid, block;
     uint32_t items = 0;
 };
-Geometry fused_geometry(const Geometry &g);  // publish_fused_kernel's grid (own occupancy)
+Geometry fused_geometry(const Geometry &g, int device);  // publish_fused_kernel's grid (own occupancy)
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms = 0);  // max_sms > 0: at most that many SMs
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
