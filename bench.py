@@ -494,6 +494,40 @@ N_CONFIG = {2: "resnet50", 4: "vit_b16", 8: "gpt2_xl"}  # BASELINE.json configs[
 CONFIG_INDEX = {"ptychonn": 0, "resnet50": 1, "vit_b16": 2, "gpt2_xl": 3, "llama3_8b": 4}
 
 
+def ce_baseline(rank, group, buf, steps, warmup):
+    """SURVEY B2 (baseline only): copy-engine delivery.  Rank 0 shares its
+    S-byte buffer through CUDA IPC (torch's own reduction), every consumer
+    copies it into a local buffer at the same time (torch copy_ across devices:
+    cudaMemcpyPeerAsync on the copy engine), device-timed per consumer.
+    Returns this rank's mean ms (0 on the producer)."""
+    import torch
+    import torch.distributed as dist
+    from torch.multiprocessing.reductions import reduce_tensor
+    obj = [reduce_tensor(buf) if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    ms = []
+    peer = local = None
+    if rank != 0:
+        fn, fargs = obj[0]
+        peer = fn(*fargs)
+        local = torch.empty_like(buf)
+    for i in range(warmup + steps):
+        torch.cuda.synchronize()
+        dist.barrier(group=group)
+        if rank != 0:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            local.copy_(peer, non_blocking=True)
+            e1.record()
+            e1.synchronize()
+            if i >= warmup:
+                ms.append(e0.elapsed_time(e1))
+    del peer, local
+    torch.cuda.synchronize()
+    dist.barrier(group=group)  # the producer's buffer outlives every mapping
+    return statistics.mean(ms) if ms else 0.0
+
+
 def xproc_e2e(V, G, synth, name, rank, world, dev, group, fanout, flush_buf, steps, warmup):
     """The N > 1 update end to end through the public API with HOST buffers
     (the N = 1 run_e2e across processes).  Rank 0's parameters live in one flat
@@ -637,11 +671,12 @@ def xproc_arm(args):
         e1.synchronize()
         if i >= args.warmup:
             nccl_ms.append(e0.elapsed_time(e1))
+    ce_ms = ce_baseline(rank, gloo, buf, args.steps, args.warmup)
     del buf
     e2e = xproc_e2e(V, G, synth, name, rank, world, dev, gloo, fanout, flush, args.steps, args.warmup)
     t = torch.tensor([statistics.mean(lat[args.warmup:]) if rank == 0 else 0.0,
                       statistics.median(inst[args.warmup:]) if rank else 0.0,
-                      statistics.mean(nccl_ms), float(1 - ok), e2e["ms"], float(1 - e2e["ok"])],
+                      statistics.mean(nccl_ms), float(1 - ok), e2e["ms"], float(1 - e2e["ok"]), ce_ms],
                      dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
     if rank != 0:
@@ -669,6 +704,10 @@ def xproc_arm(args):
                 "frac": round(S / (inst_us * 1e-6) / 1e9 / nvl, 4), "traffic": None,
                 "peak_kind": "measured peer copy (B200_PROFILING.md)"},
             "nccl_broadcast_ms": None if over else round(nccl, 6),
+            "ce_pull_ms": round(float(t[6]), 6),
+            "ce_pull_how": "SURVEY B2 baseline: every consumer pulls the producer's S bytes at once with the copy "
+                           "engine (torch copy_ from the CUDA-IPC-mapped producer buffer = cudaMemcpyPeerAsync), "
+                           "CUDA events, max over consumers",
             "parity_ok": bool(float(t[3]) == 0.0),
             "gpu_launches": 3 * args.steps,
             "clocks": clk.summary(),

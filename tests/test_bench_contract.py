@@ -12,7 +12,8 @@ sys.path.insert(0, ROOT)
 def test_bench_functions_exist():
     import bench
     for fn in ("run_update_bench", "run_e2e", "c3_concurrent", "c5_schedule", "event_floor_us", "cpu_baseline",
-               "xproc_arm", "gpu_arm", "reference_arm", "main", "ncu_traffic", "load_peaks"):
+               "xproc_arm", "xproc_e2e", "ce_baseline", "gpu_arm", "reference_arm", "main", "ncu_traffic",
+               "load_peaks"):
         assert callable(getattr(bench, fn)), fn
 
 
