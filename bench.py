@@ -138,7 +138,7 @@ class ClockSampler:
 
 # ---------------------------------------------------------------- GPU arm
 def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tier=None, kernel_timing=False,
-                     extra_flags=0):
+                     extra_flags=0, ncons=1):
     """Producer + 1 consumer on this GPU; per-step update latency.
 
     kernel_timing=False: the headline pass -- nothing but the update inside
@@ -151,12 +151,14 @@ def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tie
     specs = synth.model_specs(name)
     seed = synth.SEEDS[name]
     prod_t = G.alloc_model(specs)
-    cons_t = G.alloc_model(specs)
+    cons_ts = [G.alloc_model(specs) for _ in range(ncons)]
+    cons_t = cons_ts[0]
     mname = f"bench-{name}-{os.getpid()}-{time.monotonic_ns()}"
     flags = (V.FLAG_TIMING if kernel_timing else 0) | extra_flags
     mode = V.SYNC if mode is None else mode
     tier = V.TIER_GPU if tier is None else tier
-    cons = V.Model(mname, V.CONSUMER, cons_t, flags=flags, tier=tier)
+    conss = [V.Model(mname, V.CONSUMER, ct, flags=flags, tier=tier) for ct in cons_ts]
+    cons = conss[0]
     prod = V.Model(mname, V.PRODUCER, prod_t, flags=flags, mode=mode, tier=tier)
     st = torch.cuda.current_stream()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -185,14 +187,17 @@ def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tie
                     pack_us.append(ps["t_pack_dev_us"])
                     fused_us.append(ps["t_fused_dev_us"])
                     inst_us.append(cons.stats()["t_install_dev_us"])
-        view = cons.acquire_latest()
-        ok = view.version == warmup + steps and all(
-            torch.equal(g.view(torch.uint8), p.view(torch.uint8)) for g, p in zip(view.tensors(cons_t), prod_t))
-        cons.release(view)
+        ok = True
+        for c, ct in zip(conss, cons_ts):
+            view = c.acquire_latest()
+            ok = ok and view.version == warmup + steps and all(
+                torch.equal(g.view(torch.uint8), p.view(torch.uint8)) for g, p in zip(view.tensors(ct), prod_t))
+            c.release(view)
         s_packed = prod.stats()["s_packed"]
         nchunks = prod.stats()["nchunks"]
     finally:
-        cons.close()
+        for c in conss:
+            c.close()
         prod.close()
     return {"dev_ms": dev_ms, "host_ms": host_ms, "pack_us": pack_us, "install_us": inst_us, "fused_us": fused_us,
             "ok": ok,
@@ -827,6 +832,24 @@ def gpu_arm(args):
                     sweep[nm] = {"error": str(ex)[:200]}
                 torch.cuda.empty_cache()
             out["loopback_sweep"] = sweep
+            fan = {}
+            for nm, nc in (("vit_b16", 3), ("gpt2_xl", 3)):  # BASELINE configs[2] / [3] consumers on one GPU
+                try:
+                    s = run_update_bench(V, G, synth, nm, 5, 3, flush, ncons=nc)
+                    k = run_update_bench(V, G, synth, nm, 5, 3, flush, kernel_timing=True, ncons=nc)
+                    fu = statistics.median(k["fused_us"])
+                    lat = statistics.mean(s["dev_ms"])
+                    fan[f"{nm}_1to{nc}"] = {
+                        "latency_ms": round(lat, 4), "fused_us": round(fu, 2),
+                        "algorithmic_bytes": (2 + nc) * s["bytes"],
+                        "fused_hbm_frac": round((2 + nc) * s["bytes"] / (fu * 1e-6) / 1e9 / peak, 4),
+                        "parity_ok": s["ok"] and k["ok"]}
+                except Exception as ex:  # report, never hide
+                    fan[f"{nm}_1to{nc}"] = {"error": str(ex)[:200]}
+                torch.cuda.empty_cache()
+            out["loopback_fanout"] = {
+                "how": "in-process SYNC, 1 producer -> N consumers on this GPU: one fused kernel reads the "
+                       "tensors once and writes the snapshot + N slots ((2+N)*S bytes)", **fan}
             try:
                 out["c3_concurrent"] = c3_concurrent(V, G, synth)
                 out["c3_concurrent_gemm"] = c3_concurrent(V, G, synth, reader_kind="gemm")  # compute-bound reader
