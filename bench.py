@@ -627,8 +627,11 @@ def xproc_arm(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     gloo = dist.new_group(backend="gloo")
     bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
+    # auto: scatter-allgather for 1 -> N > 1 over NVLink; direct pulls when the
+    # ranks share GPUs (oversubscribed code-path runs: peers time-slice one GPU,
+    # so waiting on a peer's staged copy only serialises the installs)
     fanout = {"direct": V.FANOUT_DIRECT, "chain": V.FANOUT_CHAIN, "sa": V.FANOUT_SCATTER_ALLGATHER}.get(
-        args.fanout, V.FANOUT_SCATTER_ALLGATHER if world > 2 else V.FANOUT_DIRECT)
+        args.fanout, V.FANOUT_SCATTER_ALLGATHER if world > 2 and not over else V.FANOUT_DIRECT)
     fanout_name = {V.FANOUT_DIRECT: "direct pull", V.FANOUT_CHAIN: "pipelined chain",
                    V.FANOUT_SCATTER_ALLGATHER: "scatter-allgather"}[fanout]
     role = V.PRODUCER if rank == 0 else V.CONSUMER
@@ -697,7 +700,8 @@ def xproc_arm(args):
             "warmup": args.warmup, "ms_per_step": round(lat_ms, 6), "higher_is_better": False, "scaling": "weak",
             "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
             "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
-            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers over NVLink "
+            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers "
+                                   f"{'sharing one GPU (code path only, no NVLink)' if over else 'over NVLink'} "
                                    f"({fanout_name}), SYNC",
                        "model_bytes": S, "devices_visible": ndev,
                        "oversubscribed": ndev < world, "l2": "flushed before every update"},
