@@ -226,7 +226,7 @@ viper_status upload_items(const Manifest &m, const std::vector<void *> &ptrs, It
 static std::mutex g_reg_mu;
 static std::map<std::string, Channel *> g_reg;
 
-static viper_status channel_open(const std::string &name, const Manifest &man, Channel **out) {
+static viper_status channel_open(const std::string &name, const Manifest &man, int32_t tier, Channel **out) {
     std::lock_guard<std::mutex> lk(g_reg_mu);
     auto it = g_reg.find(name);
     Channel *ch;
@@ -242,11 +242,17 @@ static viper_status channel_open(const std::string &name, const Manifest &man, C
         void *d = nullptr;
         CUDA_TRY(cudaHostGetDevicePointer(&d, p, 0));
         ch->ctrl_dev = (Ctrl *)d;
+        ch->tier = tier;
         g_reg[name] = ch;
     } else {
         ch = it->second;
         if (ch->nbytes != man.nbytes)
             return set_error(VIPER_E_INVAL, "model '%s': tensor list differs from the other endpoints", name.c_str());
+        // a DRAM-tier consumer reads the producer's host staging, which only a
+        // DRAM-tier producer fills
+        if (ch->tier != tier)
+            return set_error(VIPER_E_INVAL, "model '%s': tier %d, the other endpoints use tier %d", name.c_str(), tier,
+                             ch->tier);
     }
     ch->refs++;
     *out = ch;
@@ -918,8 +924,33 @@ viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
     return VIPER_OK;
 }
 
+// In-process endpoints on two GPUs: the producer's kernels write consumer slots
+// (fused SYNC kernel, SYNC installs on the producer's stream) and a consumer's
+// kernels read the producer's snapshot, so both directions need peer access.
+// The DRAM tier moves everything through host memory and needs none.
+static viper_status link_devices(int a, int b, int32_t tier) {
+    if (a == b || tier == VIPER_TIER_DRAM) return VIPER_OK;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    viper_status st = VIPER_OK;
+    for (int k = 0; k < 2 && st == VIPER_OK; k++) {
+        const int x = k ? b : a, y = k ? a : b;
+        int can = 0;
+        if (cudaDeviceCanAccessPeer(&can, x, y) != cudaSuccess || !can) {
+            st = set_error(VIPER_E_UNSUPPORTED, "GPU tier: device %d cannot access device %d (use the DRAM tier)", x, y);
+            break;
+        }
+        cudaSetDevice(x);
+        const cudaError_t e = cudaDeviceEnablePeerAccess(y, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+        else if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "cudaDeviceEnablePeerAccess(%d -> %d): %s", x, y, cudaGetErrorString(e));
+    }
+    cudaSetDevice(cur);
+    return st;
+}
+
 static viper_status register_local(viper_model *m, const viper_tensor *tensors) {
-    viper_status st = channel_open(m->name, m->man, &m->chan);
+    viper_status st = channel_open(m->name, m->man, m->cfg.tier, &m->chan);
     if (st) return st;
     m->ctrl = m->chan->ctrl;
     m->ctrl_dev = m->chan->ctrl_dev;
@@ -927,6 +958,11 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
         viper_status ps = alloc_producer(m, tensors);
         if (ps == VIPER_OK && m->cfg.flush_dir) ps = flush_start(m, m->cfg.flush_dir);
         if (ps) return ps;
+        // chan->mu orders this against consumers registering concurrently
+        // (each side links to the endpoints it sees; lock order mu -> pmu)
+        std::lock_guard<std::mutex> ck(m->chan->mu);
+        for (viper_model *c : m->chan->consumers)
+            if ((ps = link_devices(m->device, c->device, m->cfg.tier))) return ps;
         std::lock_guard<std::mutex> lk(m->chan->pmu);  // visible only once fully built
         if (m->chan->producer) return set_error(VIPER_E_STATE, "model '%s' already has a producer", m->name.c_str());
         m->chan->producer = m;
@@ -935,6 +971,8 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
     if ((st = alloc_consumer(m, tensors))) return st;
     {
         std::lock_guard<std::mutex> lk(m->chan->mu);
+        if (viper_model *p = channel_producer(m->chan))
+            if ((st = link_devices(p->device, m->device, m->cfg.tier))) return st;
         const int idx = m->ctrl->ncons.load();
         if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
         m->cidx = idx;

@@ -209,6 +209,7 @@ struct Channel {
     std::vector<viper_model *> consumers;
     int refs = 0;
     std::vector<uint64_t> nbytes;  // manifest check
+    int32_t tier = -1;             // every endpoint of an in-process channel uses one tier
 };
 
 struct PreparedInstall {

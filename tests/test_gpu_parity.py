@@ -179,6 +179,37 @@ def test_empty_model():
         close_all(prod, [cons])
 
 
+# ------------------------------------------------------ in-process tier agreement
+@pytest.mark.parametrize("first,second", [(V.TIER_GPU, V.TIER_DRAM), (V.TIER_DRAM, V.TIER_GPU)])
+def test_in_process_endpoints_must_share_a_tier(first, second):
+    """A DRAM-tier consumer reads the producer's host staging, which a GPU-tier
+    producer never fills: registration with mixed tiers is refused (E_INVAL),
+    whichever side registers first, and the channel stays usable."""
+    specs = synth.model_specs("ptychonn")
+    seed = synth.SEEDS["ptychonn"]
+    name = uname()
+    pt, ct, ct2 = G.alloc_model(specs), G.alloc_model(specs), G.alloc_model(specs)
+    cons = V.Model(name, V.CONSUMER, ct, tier=first)
+    try:
+        with pytest.raises(V.ViperError) as ei:
+            V.Model(name, V.PRODUCER, pt, tier=second)
+        assert ei.value.status == V.E_INVAL
+        with pytest.raises(V.ViperError) as ei:
+            V.Model(name, V.CONSUMER, ct2, tier=second)
+        assert ei.value.status == V.E_INVAL
+        prod = V.Model(name, V.PRODUCER, pt, tier=first)
+        try:
+            G.fill_model(pt, specs, seed, 1)
+            prod.publish(1)
+            view = cons.acquire_latest(min_version=1, timeout_us=5_000_000)
+            check_slot(view, ct, specs, seed, 1)
+            cons.release(view)
+        finally:
+            prod.close()
+    finally:
+        cons.close()
+
+
 # ---------------------------------------------------------------- protocol on device
 @pytest.mark.parametrize("flags", [0, V.FLAG_NO_FUSE, V.FLAG_FUSED_TMA, V.FLAG_NO_TMA])
 def test_fault_injection_keeps_old_version(flags):
