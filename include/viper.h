@@ -91,7 +91,17 @@ typedef struct {
 
 /* Storage tier (s4.4 P:1671-1720, Fig. 7). */
 enum { VIPER_TIER_GPU = 0,   /* GPU-to-GPU memory: pull over NVLink peer mapping */
-       VIPER_TIER_DRAM = 1 }; /* Host-to-Host memory: staged through pinned DRAM  */
+       VIPER_TIER_DRAM = 1,  /* Host-to-Host memory: staged through pinned DRAM  */
+       VIPER_TIER_AUTO = 2 }; /* Transfer Selector (Fig. 7): decided
+                                once at registration, the same on every endpoint.
+                                Cross-process: the GPU tier when every consumer's
+                                GPU can peer-access every producer's GPU (or is
+                                the same GPU), else the DRAM tier; every rank
+                                must then ask for AUTO.  In process: the tier of
+                                the model's existing endpoints, else the GPU tier
+                                when this GPU can peer-access every visible GPU
+                                (or is the only one).  viper_stats.tier reports
+                                the choice. */
 /* Fan-out of one producer to N consumers. */
 enum { VIPER_FANOUT_DIRECT = 0,        /* every consumer pulls every chunk from the producer */
        VIPER_FANOUT_CHAIN = 1,         /* pipelined chain: consumer i pulls every item from
@@ -253,6 +263,8 @@ typedef struct {
     int32_t last_status;
     int32_t nconsumers;
     uint64_t flushed, flush_skipped, flush_last;  /* producer with flush_dir        */
+    int32_t tier;              /* tier in use (VIPER_TIER_AUTO resolved)               */
+    int32_t fanout;            /* fan-out in use                                       */
 } viper_stats;
 viper_status viper_get_stats(viper_model *m, viper_stats *out);
 

@@ -949,7 +949,27 @@ static viper_status link_devices(int a, int b, int32_t tier) {
     return st;
 }
 
+// Transfer Selector, in process (VIPER_TIER_AUTO): the tier of the model's
+// existing endpoints; for the first one, the GPU tier when this GPU can
+// peer-access every visible GPU (or is the only one) -- a process-wide fact,
+// so endpoints registering concurrently decide alike -- else the DRAM tier.
+static int32_t select_tier_local(const std::string &name, int device) {
+    {
+        std::lock_guard<std::mutex> lk(g_reg_mu);
+        auto it = g_reg.find(name);
+        if (it != g_reg.end()) return it->second->tier;
+    }
+    int ndev = 0;
+    cudaGetDeviceCount(&ndev);
+    for (int d = 0; d < ndev; d++) {
+        int can = 0;
+        if (d != device && (cudaDeviceCanAccessPeer(&can, device, d) != cudaSuccess || !can)) return VIPER_TIER_DRAM;
+    }
+    return VIPER_TIER_GPU;
+}
+
 static viper_status register_local(viper_model *m, const viper_tensor *tensors) {
+    if (m->cfg.tier == VIPER_TIER_AUTO) m->cfg.tier = select_tier_local(m->name, m->device);
     viper_status st = channel_open(m->name, m->man, m->cfg.tier, &m->chan);
     if (st) return st;
     m->ctrl = m->chan->ctrl;
@@ -1029,7 +1049,8 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
         if (c.align == 0) c.align = 256;
         if (c.align < 16 || (c.align & (c.align - 1))) return set_error(VIPER_E_INVAL, "align must be a power of 2 >= 16");
         if (c.chunk_bytes % 256 || c.chunk_bytes % c.align) return set_error(VIPER_E_INVAL, "chunk_bytes must be a multiple of 256 and align");
-        if (c.tier != VIPER_TIER_GPU && c.tier != VIPER_TIER_DRAM) return set_error(VIPER_E_INVAL, "bad tier");
+        if (c.tier != VIPER_TIER_GPU && c.tier != VIPER_TIER_DRAM && c.tier != VIPER_TIER_AUTO)
+            return set_error(VIPER_E_INVAL, "bad tier");
         if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
         if (c.install_sms < 0) return set_error(VIPER_E_INVAL, "install_sms must be >= 0");
         if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_CHAIN &&
@@ -1217,6 +1238,8 @@ viper_status viper_get_stats(viper_model *m, viper_stats *out) {
     *out = m->stats;
     out->nconsumers = m->ctrl ? m->ctrl->ncons.load() : 0;
     flush_stats(m, &out->flushed, &out->flush_skipped, &out->flush_last);
+    out->tier = m->cfg.tier;
+    out->fanout = m->cfg.fanout;
     return VIPER_OK;
 }
 

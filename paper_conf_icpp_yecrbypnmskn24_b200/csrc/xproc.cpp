@@ -34,6 +34,18 @@ namespace vp {
 namespace {
 
 constexpr uint32_t kPeerMagic = 0x56495052u;  // "VIPR"
+constexpr uint32_t kTierMagic = 0x56495452u;  // "VITR"
+constexpr int kMaxReach = 16;
+
+// Transfer Selector round (the first bootstrap allgather, every rank): the
+// tier asked for and the GPUs this rank's GPU can reach (itself included), as
+// PCI bus ids, so that every rank resolves VIPER_TIER_AUTO from the same data.
+struct TierRec {
+    uint32_t magic;
+    int32_t tier, nreach, pad;
+    char pci[16];
+    char reach[kMaxReach][16];
+};
 
 struct PeerRec {
     uint32_t magic;
@@ -209,6 +221,43 @@ viper_status open_producers(viper_model *m, const std::vector<PeerRec> &all, con
     return VIPER_OK;
 }
 
+// Pre-round of the bootstrap: VIPER_TIER_AUTO -> GPU when every consumer's
+// GPU reaches every producer's GPU (same GPU or peer access), else DRAM.
+// Records of ranks that failed before the bootstrap (magic 0) decide nothing:
+// those ranks fail the registration in the next round anyway.
+// VIPER_TEST_NO_PEER=1 (tests): this rank reports that it reaches no GPU.
+int32_t select_tier_xproc(const viper_model *m, const viper_bootstrap *bs, int M, bool *comm_ok) {
+    TierRec me{};
+    me.magic = kTierMagic;
+    me.tier = m->cfg.tier;
+    cudaDeviceGetPCIBusId(me.pci, sizeof me.pci, m->device);
+    const char *hook = getenv("VIPER_TEST_NO_PEER");
+    if (!(hook && atoi(hook))) {
+        memcpy(me.reach[me.nreach++], me.pci, sizeof me.pci);
+        int ndev = 0;
+        cudaGetDeviceCount(&ndev);
+        for (int d = 0; d < ndev && me.nreach < kMaxReach; d++) {
+            int can = 0;
+            if (d == m->device || cudaDeviceCanAccessPeer(&can, m->device, d) != cudaSuccess || !can) continue;
+            cudaDeviceGetPCIBusId(me.reach[me.nreach++], 16, d);
+        }
+    }
+    std::vector<TierRec> all(bs->world);
+    *comm_ok = bs->allgather(&me, all.data(), sizeof(TierRec), bs->user) == 0;
+    if (!*comm_ok || m->cfg.tier != VIPER_TIER_AUTO) return m->cfg.tier;
+    for (int c = 0; c < bs->world; c++) {
+        if (c >= bs->producer_rank && c < bs->producer_rank + M) continue;  // a producer
+        for (int p = bs->producer_rank; p < bs->producer_rank + M; p++) {
+            if (all[c].magic != kTierMagic || all[p].magic != kTierMagic) continue;
+            bool ok = false;
+            for (int k = 0; k < all[c].nreach && k < kMaxReach && !ok; k++)
+                ok = strncmp(all[c].reach[k], all[p].pci, 16) == 0;
+            if (!ok) return VIPER_TIER_DRAM;
+        }
+    }
+    return VIPER_TIER_GPU;
+}
+
 }  // namespace
 
 viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const viper_bootstrap *bs) {
@@ -225,6 +274,9 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         xproc_abort(bs, bad);  // (does not touch the error text)
         return bad;
     }
+    bool comm_ok = true;
+    m->cfg.tier = select_tier_xproc(m, bs, M, &comm_ok);  // Transfer Selector
+    if (!comm_ok) return set_error(VIPER_E_PEER, "bootstrap allgather failed");
     m->rank = bs->rank;
     m->world = bs->world;
     m->nconsumers_x = bs->world - M;
@@ -378,6 +430,11 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
 }
 
 void xproc_abort(const viper_bootstrap *bs, viper_status st) {
+    {
+        TierRec t{};  // the Transfer Selector round (magic 0: decides nothing)
+        std::vector<TierRec> tall(bs->world > 0 ? bs->world : 1);
+        if (bs->allgather(&t, tall.data(), sizeof(TierRec), bs->user) != 0) return;
+    }
     PeerRec me{};
     me.magic = kPeerMagic;
     me.rank = bs->rank;

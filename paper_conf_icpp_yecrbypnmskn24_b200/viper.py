@@ -16,7 +16,7 @@ OK, E_INVAL, E_NOMEM, E_CUDA, E_VERSION, E_CHECKSUM, E_TIMEOUT, E_NOVERSION, E_S
     0, -1, -2, -3, -4, -5, -6, -7, -8, -9, -10)
 PRODUCER, CONSUMER = 1, 2
 F32, BF16, F16, BYTES = 0, 1, 2, 3
-TIER_GPU, TIER_DRAM = 0, 1
+TIER_GPU, TIER_DRAM, TIER_AUTO = 0, 1, 2
 FANOUT_DIRECT, FANOUT_CHAIN, FANOUT_SCATTER_ALLGATHER = 0, 1, 2
 SYNC, ASYNC = 0, 1
 FLAG_TIMING = 2
@@ -57,7 +57,8 @@ class viper_stats(C.Structure):
                 ("t_publish_us", C.c_double), ("t_install_us", C.c_double), ("t_notify_us", C.c_double),
                 ("writer_wait_us", C.c_double), ("t_pack_dev_us", C.c_double),
                 ("t_install_dev_us", C.c_double), ("t_fused_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32),
-                ("flushed", C.c_uint64), ("flush_skipped", C.c_uint64), ("flush_last", C.c_uint64)]
+                ("flushed", C.c_uint64), ("flush_skipped", C.c_uint64), ("flush_last", C.c_uint64),
+                ("tier", C.c_int32), ("fanout", C.c_int32)]
 
 
 class viper_sched_in(C.Structure):

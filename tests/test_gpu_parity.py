@@ -210,6 +210,33 @@ def test_in_process_endpoints_must_share_a_tier(first, second):
         cons.close()
 
 
+@pytest.mark.parametrize("first", [V.TIER_AUTO, V.TIER_DRAM, V.TIER_GPU])
+def test_in_process_transfer_selector(first):
+    """VIPER_TIER_AUTO in process: the tier of the model's existing endpoints,
+    else the GPU tier when this GPU reaches every visible GPU (here: the only
+    one).  The producer registers with AUTO after a consumer asked for
+    `first`; both report the same resolved tier and the update is bit-exact."""
+    import torch
+    specs = synth.model_specs("ptychonn")
+    seed = synth.SEEDS["ptychonn"]
+    name = uname()
+    pt, ct = G.alloc_model(specs), G.alloc_model(specs)
+    cons = V.Model(name, V.CONSUMER, ct, tier=first)
+    prod = V.Model(name, V.PRODUCER, pt, tier=V.TIER_AUTO)
+    try:
+        solo = torch.cuda.device_count() == 1
+        want = first if first != V.TIER_AUTO else (V.TIER_GPU if solo else cons.stats()["tier"])
+        assert cons.stats()["tier"] == want and prod.stats()["tier"] == want
+        for v in (1, 2):
+            G.fill_model(pt, specs, seed, v)
+            prod.publish(v)
+        view = cons.acquire_latest(min_version=2, timeout_us=5_000_000)
+        check_slot(view, ct, specs, seed, 2)
+        cons.release(view)
+    finally:
+        close_all(prod, [cons])
+
+
 # ---------------------------------------------------------------- protocol on device
 @pytest.mark.parametrize("flags", [0, V.FLAG_NO_FUSE, V.FLAG_FUSED_TMA, V.FLAG_NO_TMA])
 def test_fault_injection_keeps_old_version(flags):

@@ -82,6 +82,10 @@ def main():
     ap.add_argument("--delay-ms", type=float, default=0.0,
                     help="ASYNC: the producer's stream sleeps this long before each publish; consumers check "
                          "that their install did not start (and spin) before the stream reached the pack")
+    ap.add_argument("--expect-tier", type=int, default=-1, help="check the tier in use after registration "
+                    "(VIPER_TIER_AUTO resolved by the Transfer Selector)")
+    ap.add_argument("--no-peer-rank", type=int, default=-1, help="this rank reports that it reaches no GPU "
+                    "(VIPER_TEST_NO_PEER)")
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
@@ -94,9 +98,14 @@ def main():
     bs = V.Bootstrap(rank, world, producer_rank=0, nproducers=a.nprod)
     is_prod = rank < a.nprod
     role = V.PRODUCER if is_prod else V.CONSUMER
+    if rank == a.no_peer_rank:
+        os.environ["VIPER_TEST_NO_PEER"] = "1"
     m = V.Model(f"xp-{a.config}", role, tensors, tier=a.tier, mode=a.mode, fanout=a.fanout, device=dev,
                 bootstrap=bs)
     errors = 0
+    if a.expect_tier >= 0 and m.stats()["tier"] != a.expect_tier:
+        print(f"[rank{rank}] tier {m.stats()['tier']}, want {a.expect_tier}", flush=True)
+        errors += 1
     last = 0
     if a.stress:
         errors += stress(m, rank, specs, seed, tensors, a.versions, dev)
