@@ -95,8 +95,10 @@ enum { VIPER_TIER_GPU = 0,   /* GPU-to-GPU memory: pull over NVLink peer mapping
        VIPER_TIER_AUTO = 2 }; /* Transfer Selector (Fig. 7): decided
                                 once at registration, the same on every endpoint.
                                 Cross-process: the GPU tier when every consumer's
-                                GPU can peer-access every producer's GPU (or is
-                                the same GPU), else the DRAM tier; every rank
+                                GPU can peer-access every producer's GPU (and,
+                                with chain / scatter-allgather fan-out, every
+                                other consumer's; or is the same GPU), else the
+                                DRAM tier; every rank
                                 must then ask for AUTO.  In process: the tier of
                                 the model's existing endpoints, else the GPU tier
                                 when this GPU can peer-access every visible GPU

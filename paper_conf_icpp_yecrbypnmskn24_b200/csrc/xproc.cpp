@@ -245,15 +245,20 @@ int32_t select_tier_xproc(const viper_model *m, const viper_bootstrap *bs, int M
     std::vector<TierRec> all(bs->world);
     *comm_ok = bs->allgather(&me, all.data(), sizeof(TierRec), bs->user) == 0;
     if (!*comm_ok || m->cfg.tier != VIPER_TIER_AUTO) return m->cfg.tier;
+    auto producer = [&](int r) { return r >= bs->producer_rank && r < bs->producer_rank + M; };
+    auto reaches = [&](int a, int b) {  // rank a's GPU can read rank b's GPU memory
+        if (all[a].magic != kTierMagic || all[b].magic != kTierMagic) return true;
+        for (int k = 0; k < all[a].nreach && k < kMaxReach; k++)
+            if (strncmp(all[a].reach[k], all[b].pci, 16) == 0) return true;
+        return false;
+    };
+    // consumers pull from the producers, and with chain / scatter-allgather
+    // fan-out also from each other
+    const bool peers = m->cfg.fanout == VIPER_FANOUT_CHAIN || m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER;
     for (int c = 0; c < bs->world; c++) {
-        if (c >= bs->producer_rank && c < bs->producer_rank + M) continue;  // a producer
-        for (int p = bs->producer_rank; p < bs->producer_rank + M; p++) {
-            if (all[c].magic != kTierMagic || all[p].magic != kTierMagic) continue;
-            bool ok = false;
-            for (int k = 0; k < all[c].nreach && k < kMaxReach && !ok; k++)
-                ok = strncmp(all[c].reach[k], all[p].pci, 16) == 0;
-            if (!ok) return VIPER_TIER_DRAM;
-        }
+        if (producer(c)) continue;
+        for (int r = 0; r < bs->world; r++)
+            if (r != c && (producer(r) || peers) && !reaches(c, r)) return VIPER_TIER_DRAM;
     }
     return VIPER_TIER_GPU;
 }

@@ -51,9 +51,10 @@ def test_xproc_scatter_allgather(nproc, mode, config):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("nproc,mode,no_peer_rank,expect", [(3, 0, -1, 0), (3, 1, -1, 0), (3, 0, 2, 1),
-                                                           (2, 1, 1, 1), (2, 0, 0, 0)])
-def test_xproc_transfer_selector(nproc, mode, no_peer_rank, expect):
+@pytest.mark.parametrize("nproc,mode,fanout,no_peer_rank,expect", [
+    (3, 0, 0, -1, 0), (3, 1, 0, -1, 0), (3, 0, 0, 2, 1), (2, 1, 0, 1, 1), (2, 0, 0, 0, 0),
+    (4, 0, 2, -1, 0), (4, 0, 2, 3, 1), (3, 1, 1, 1, 1)])
+def test_xproc_transfer_selector(nproc, mode, fanout, no_peer_rank, expect):
     """VIPER_TIER_AUTO (Transfer Selector): every rank resolves the
     same tier from the bootstrap's reachability round -- GPU while every consumer
     reaches the producer's GPU, DRAM as soon as one rank reports it cannot
@@ -61,7 +62,8 @@ def test_xproc_transfer_selector(nproc, mode, no_peer_rank, expect):
     producer's own reach does not matter: consumers pull from it."""
     rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
                            ["--config", "small", "--tier", "2", "--mode", str(mode), "--versions", "4",
-                            "--expect-tier", str(expect), "--no-peer-rank", str(no_peer_rank)])
+                            "--expect-tier", str(expect), "--no-peer-rank", str(no_peer_rank),
+                            "--fanout", str(fanout)])
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
 
 
