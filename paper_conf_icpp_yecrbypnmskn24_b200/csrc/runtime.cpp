@@ -334,9 +334,11 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
             if (s) return s;
             CUDA_TRY(cudaMemcpyAsync(c->d_stage + mm.piece_lo[i], src.h_stage[b] + mm.piece_lo[i],
                                      mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyHostToDevice, st));
-            CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal + mm.piece_ilo[i], src.h_iseal[b] + mm.piece_ilo[i],
-                                     sizeof(ISeal) * (mm.piece_ihi[i] - mm.piece_ilo[i]), cudaMemcpyHostToDevice, st));
         }
+        // the item seals travel once, behind the last piece (the producer
+        // raises the last flag after their D2H); only the install reads them
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.h_iseal[b], sizeof(ISeal) * mm.items.size(),
+                                 cudaMemcpyHostToDevice, st));
         pdl = false;
     } else if (wait_ready && src.ev_ready[b]) {
         CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
@@ -722,12 +724,13 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // stream (the caller's stream is blocked only by the pack); each piece
         // raises its flag for the consumers' H2D
         const Manifest &mm = p->man;
-        for (size_t i = 0; i < mm.piece_lo.size(); i++) {
+        const size_t np = mm.piece_lo.size();
+        for (size_t i = 0; i < np; i++) {
             CUDA_TRY(cudaMemcpyAsync(p->h_stage[b] + mm.piece_lo[i], p->d_snap[b] + mm.piece_lo[i],
                                      mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyDeviceToHost, p->side));
-            CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b] + mm.piece_ilo[i], p->d_iseal[b] + mm.piece_ilo[i],
-                                     sizeof(ISeal) * (mm.piece_ihi[i] - mm.piece_ilo[i]), cudaMemcpyDeviceToHost,
-                                     p->side));
+            if (i + 1 == np)  // item seals once, before the last flag (one copy instead of one per piece)
+                CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b], p->d_iseal[b], sizeof(ISeal) * mm.items.size(),
+                                         cudaMemcpyDeviceToHost, p->side));
             viper_status s = stream_write(p->side, &p->ctrl_dev->dram_flag[b][i], v);
             if (s) return s;
         }
