@@ -19,6 +19,8 @@ def lib():
         _lib.vgen_fill.restype = C.c_int
         _lib.l2_flush.argtypes = [C.c_void_p, C.c_uint64, C.c_void_p]
         _lib.l2_flush.restype = C.c_int
+        _lib.l2_flush_clean.argtypes = [C.c_void_p, C.c_uint64, C.c_void_p]
+        _lib.l2_flush_clean.restype = C.c_int
         _lib.launch_empty.argtypes = [C.c_void_p]
         _lib.launch_empty.restype = C.c_int
         _lib.host_alloc.argtypes = [C.c_uint64]
@@ -56,8 +58,14 @@ def alloc_model(specs, device=None):
     return [torch.empty(s[2], dtype=dt.get(s[1], torch.uint8), device=device) for s in specs]
 
 
-def l2_flush(buf, stream=None):
-    if lib().l2_flush(C.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(), _sp(stream)) != 0:
+def l2_flush(buf, stream=None, clean=False):
+    """Evict L2 between timed steps by writing `buf` (> L2).  clean=True: write
+    its first half, then read its second half (each half > L2), so the dirty
+    lines are written back inside the flush and L2 holds clean unrelated data
+    (ncu's cache-control state) instead of ~126 MB of dirty harness lines that
+    the next kernel would have to write back."""
+    fn = lib().l2_flush_clean if clean else lib().l2_flush
+    if fn(C.c_void_p(buf.data_ptr()), buf.numel() * buf.element_size(), _sp(stream)) != 0:
         raise RuntimeError("l2_flush failed")
 
 

@@ -73,6 +73,31 @@ extern "C" int l2_flush(void *dev_ptr, uint64_t bytes, void *stream) {
     return cudaMemsetAsync(dev_ptr, (int)(bytes & 0xFF), bytes, (cudaStream_t)stream) == cudaSuccess ? 0 : -3;
 }
 
+namespace {
+__global__ void l2_read_kernel(const uint4 *p, uint64_t n, uint32_t *sink) {
+    uint32_t x = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 v = __ldcg(p + i);
+        x ^= v.x ^ v.y ^ v.z ^ v.w;
+    }
+    if (x == 0x9E3779B9u) *sink = x;  // keeps the loads; never true for the memset pattern
+}
+}  // namespace
+
+// Clean flush: write the first half of the buffer (each half > L2), then read
+// the second half, so the first half's dirty lines are written back HERE and
+// L2 ends up holding clean, unrelated lines -- the state ncu's cache control
+// leaves before a kernel.  The timed kernel then pays no write-back of
+// harness data.
+extern "C" int l2_flush_clean(void *dev_ptr, uint64_t bytes, void *stream) {
+    const uint64_t half = bytes / 2 / 16 * 16;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (cudaMemsetAsync(dev_ptr, 0x5A, half, st) != cudaSuccess) return -3;
+    uint8_t *second = (uint8_t *)dev_ptr + half;
+    l2_read_kernel<<<148 * 4, 512, 0, st>>>((const uint4 *)second, half / 16, (uint32_t *)second);
+    return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+
 // Harness helpers for bench.py's e2e leg: pinned host buffers and copies
 // through the CUDA runtime directly (torch's pinned copy path measured
 // erratic H2D throughput on this VM, profiles/r01/h2dcal.log).

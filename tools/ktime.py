@@ -21,7 +21,7 @@ a = ap.parse_args()
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
-flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")  # --flush 1: write 256 MiB; 2: + read 256 MiB
 S = synth.model_bytes(a.config)
 res = {}
 for label, flags in (("fused", V.FLAG_NO_TMA), ("fused_tma", V.FLAG_FUSED_TMA), ("sep", V.FLAG_NO_FUSE | V.FLAG_NO_TMA),
@@ -33,8 +33,10 @@ for label, flags in (("fused", V.FLAG_NO_TMA), ("fused_tma", V.FLAG_FUSED_TMA), 
     fu, pk, ins = [], [], []
     for v in range(1, a.steps + 4):
         G.fill_model(pt, specs, seed, v, stream=st)
-        if a.flush:
-            G.l2_flush(flush, stream=st)
+        if a.flush == 1:
+            G.l2_flush(flush[:256 << 20], stream=st)
+        elif a.flush == 2:
+            G.l2_flush(flush, stream=st, clean=True)
         torch.cuda._sleep(400_000)
         p.publish(v, stream=st)
         torch.cuda.synchronize()
