@@ -21,6 +21,7 @@ ap.add_argument("--config", default="resnet50")
 ap.add_argument("--steps", type=int, default=5)
 ap.add_argument("--defines", default="")
 ap.add_argument("--lib", default=LIBP)
+ap.add_argument("--clean", action="store_true", help="write + read L2 flush (bench.py default)")
 a = ap.parse_args()
 if a.build:
     from paper_conf_icpp_yecrbypnmskn24_b200 import build as B
@@ -37,7 +38,7 @@ from synth import gpu as G
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
-flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 lib = C.CDLL(a.lib)
 lib.vp_debug_warp_prof.argtypes = [C.c_void_p, C.c_int]
 NW = 296 * 8
@@ -47,7 +48,7 @@ st = torch.cuda.current_stream()
 rows = []
 for v in range(1, a.steps + 4):
     G.fill_model(pt, specs, seed, v, stream=st)
-    G.l2_flush(flush, stream=st)
+    G.l2_flush(flush if a.clean else flush[:256 << 20], stream=st, clean=a.clean)
     torch.cuda._sleep(400_000)
     buf = np.zeros(NW * 4 + 1, dtype=np.uint64)
     p.publish(v, stream=st)
