@@ -708,6 +708,11 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // in process, consumers order themselves after ev_ready[b]
         pub_word(p).store((v << 1) | (uint64_t)b);
         ctrl->pub_time_ns.store(now_ns());
+        if (!sync) {  // ASYNC: wake the update threads now; their installs wait on ev_ready[b] (and,
+                      // DRAM tier, on the pieces' flags) on the GPU, so the rest of this call overlaps them
+            ctrl->pub_seq.fetch_add(1);
+            futex_wake_all(&ctrl->pub_seq);
+        }
     }
     // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
@@ -774,9 +779,6 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         TRACE(6);
         locks.clear();
         for (viper_model *c : launched) fire_callback(c, v, c->rec->last_status.load());
-    } else {
-        ctrl->pub_seq.fetch_add(1);
-        futex_wake_all(&ctrl->pub_seq);
     }
     {
         std::lock_guard<std::mutex> lk(p->stats_mu);
