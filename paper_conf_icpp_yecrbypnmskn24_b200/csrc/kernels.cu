@@ -1133,6 +1133,31 @@ cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device
     return cudaGetLastError();
 }
 
+LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int device) {
+    LaunchSpec l{};
+    if (tma) {
+        static std::atomic<uint64_t> opted{0};
+        l.func = (const void *)pack_seal_tma_kernel;
+        l.err = opt_in_smem(pack_seal_tma_kernel, kTmaSmem, device, opted);
+        l.grid = grid_for(a.nitems, kTmaWarps, sm_count(device), 2);
+        l.block = kTmaWarps * 32;
+        l.smem = kTmaSmem;
+    } else {
+        l.func = (const void *)pack_seal_kernel;
+        l.grid = g.grid;
+        l.block = g.block;
+    }
+    return l;
+}
+
+LaunchSpec seal_reduce_launch(const SealReduceArgs &a) {
+    LaunchSpec l{};
+    l.func = (const void *)seal_reduce_kernel;
+    l.grid = (int)((a.nchunks + 7) / 8);
+    l.block = 256;
+    return l;
+}
+
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st) {
     if (a.nchunks == 0) return cudaSuccess;
     seal_reduce_kernel<<<(a.nchunks + 7) / 8, 256, 0, st>>>(a);

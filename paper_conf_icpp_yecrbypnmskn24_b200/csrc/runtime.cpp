@@ -523,11 +523,51 @@ int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug
 static const bool g_trace_on = getenv("VIPER_TRACE") != nullptr;  // tools/trace_publish.py sets it
 #define TRACE(i) (g_trace_on ? (void)(g_trace[i] = now_ns()) : (void)0)
 
-// The fused kernel through a one-node CUDA graph whose parameters are updated
-// per publish: measured cheaper on the host than a direct launch
-// (profiles/r01/launchcal.log).  VIPER_NO_GRAPH=1 launches directly.
+cudaError_t OneNodeGraph::launch(const cudaKernelNodeParams &kp, cudaStream_t st) {
+    cudaError_t e;
+    if (x && func != kp.func) destroy();
+    if (!x) {
+        if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
+        if ((e = cudaGraphAddKernelNode(&n, g, nullptr, 0, &kp)) != cudaSuccess) return e;
+        if ((e = cudaGraphInstantiate(&x, g, 0)) != cudaSuccess) return e;
+        func = kp.func;
+    } else if ((e = cudaGraphExecKernelNodeSetParams(x, n, &kp)) != cudaSuccess) {
+        return e;
+    }
+    return cudaGraphLaunch(x, st);
+}
+
+void OneNodeGraph::destroy() {
+    if (x) cudaGraphExecDestroy(x);
+    if (g) cudaGraphDestroy(g);
+    x = nullptr;
+    g = nullptr;
+    n = nullptr;
+    func = nullptr;
+}
+
+static const bool g_no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));  // direct launches
+
+// A LaunchSpec with one by-value argument struct, through a one-node graph
+// (or directly with VIPER_NO_GRAPH=1).
+template <typename Args>
+static cudaError_t launch_spec(OneNodeGraph &og, const LaunchSpec &l, const Args &a, cudaStream_t st) {
+    if (l.err != cudaSuccess) return l.err;
+    void *args[] = {(void *)&a};
+    if (g_no_graph) return cudaLaunchKernel(l.func, dim3(l.grid), dim3(l.block), args, l.smem, st);
+    cudaKernelNodeParams kp{};
+    kp.func = (void *)l.func;
+    kp.gridDim = dim3(l.grid);
+    kp.blockDim = dim3(l.block);
+    kp.sharedMemBytes = (unsigned)l.smem;
+    kp.kernelParams = args;
+    return og.launch(kp, st);
+}
+
+// The fused kernel through its one-node graph: measured cheaper on the host
+// than a direct launch (profiles/r01/launchcal.log).
 static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStream_t st) {
-    static const bool no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));
+    const bool no_graph = g_no_graph;
     static const int tma_env = getenv("VIPER_FUSED_TMA") ? atoi(getenv("VIPER_FUSED_TMA")) : -1;
     const int32_t fl = p->cfg.flags;
     const bool tma = tma_env >= 0                  ? tma_env != 0
@@ -552,15 +592,7 @@ static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStr
         kp.blockDim = dim3(fg.block);
     }
     kp.kernelParams = args;
-    cudaError_t e;
-    if (!p->fused_exec) {
-        if ((e = cudaGraphCreate(&p->fused_graph, 0)) != cudaSuccess) return e;
-        if ((e = cudaGraphAddKernelNode(&p->fused_node, p->fused_graph, nullptr, 0, &kp)) != cudaSuccess) return e;
-        if ((e = cudaGraphInstantiate(&p->fused_exec, p->fused_graph, 0)) != cudaSuccess) return e;
-    } else if ((e = cudaGraphExecKernelNodeSetParams(p->fused_exec, p->fused_node, &kp)) != cudaSuccess) {
-        return e;
-    }
-    return cudaGraphLaunch(p->fused_exec, st);
+    return p->g_fused.launch(kp, st);
 }
 
 std::atomic<uint64_t> &pub_word(viper_model *p) {
@@ -678,8 +710,11 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         a.version = v;
         a.sys_release = p->early_notify ? 1u : 0u;
         if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
-        if (tma) CUDA_TRY(launch_pack_tma(a, st, p->device));
-        else CUDA_TRY(launch_pack(a, p->geo, st));
+        // a PDL-chained install must follow a plain stream launch; every
+        // other pack goes through its one-node graph (cheaper on the host)
+        const bool pdl_follows = sync && !dram && !tma && !prepared.empty();
+        if (pdl_follows) CUDA_TRY(launch_pack(a, p->geo, st));
+        else if (a.nitems) CUDA_TRY(launch_spec(p->g_pack, pack_launch(a, p->geo, tma, p->device), a, st));
         if (timing) {
             CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
             p->timing_pending = true;
@@ -750,7 +785,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     ra.version = v;
     ra.share_n = (uint32_t)p->nprod;
     ra.share_me = (uint32_t)p->pidx;
-    CUDA_TRY(launch_seal_reduce(ra, p->side));
+    if (ra.nchunks) CUDA_TRY(launch_spec(p->g_seal, seal_reduce_launch(ra), ra, p->side));
     if (p->flusher) {  // background flush of this version, off the training stream
         viper_status s = flush_enqueue(p, v, b);
         if (s) return s;
@@ -851,8 +886,9 @@ static void free_model(viper_model *m) {
             if (evs[k]) cudaEventDestroy(evs[k]);
     if (m->ev_packed) cudaEventDestroy(m->ev_packed);
     if (m->ev_notify) cudaEventDestroy(m->ev_notify);
-    if (m->fused_exec) cudaGraphExecDestroy(m->fused_exec);
-    if (m->fused_graph) cudaGraphDestroy(m->fused_graph);
+    m->g_fused.destroy();
+    m->g_pack.destroy();
+    m->g_seal.destroy();
     if (m->side) cudaStreamDestroy(m->side);
     if (m->ustream) cudaStreamDestroy(m->ustream);
     delete m;

@@ -88,6 +88,19 @@ struct Manifest {
 struct Channel;
 struct Flusher;
 
+// One kernel launched through a one-node CUDA graph whose node parameters are
+// updated per launch: measured cheaper on the host than a direct launch on
+// this VM (profiles/r01/launchcal.log: 2.3 vs 4.5 us).  The graph is rebuilt
+// when the kernel function changes.
+struct OneNodeGraph {
+    cudaGraph_t g = nullptr;
+    cudaGraphExec_t x = nullptr;
+    cudaGraphNode_t n = nullptr;
+    const void *func = nullptr;
+    cudaError_t launch(const cudaKernelNodeParams &kp, cudaStream_t st);
+    void destroy();
+};
+
 // Where a consumer reads snapshot slot b from: the producer's device buffers
 // (same process, or CUDA-IPC peer-mapped over NVLink), the host staging of the
 // DRAM tier (pinned; a shared-memory segment across processes), and -- in
@@ -134,9 +147,7 @@ struct viper_model {
     cudaEvent_t ev_t[2] = {nullptr, nullptr};        // VIPER_FLAG_TIMING: around the kernel
     bool timing_pending = false;
     bool last_fused = false;                         // last publish used publish_fused_kernel
-    cudaGraph_t fused_graph = nullptr;               // one-node graph: cheaper per-publish launch
-    cudaGraphExec_t fused_exec = nullptr;
-    cudaGraphNode_t fused_node = nullptr;
+    vp::OneNodeGraph g_fused, g_pack, g_seal;        // per-publish launches through one-node graphs
     cudaStream_t side = nullptr;                     // DRAM-tier D2H stream
     uint8_t *h_stage[2] = {nullptr, nullptr};        // DRAM tier (pinned)
     vp::ISeal *h_iseal[2] = {nullptr, nullptr};

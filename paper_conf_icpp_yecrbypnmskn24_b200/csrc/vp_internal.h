@@ -139,15 +139,20 @@ cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
 const void *fused_kernel_fn();  // for the one-node launch graph (runtime.cpp)
-// TMA bulk-copy variant of the fused kernel: function, geometry and dynamic
-// shared memory for the launch graph (err != cudaSuccess: not launchable)
-struct FusedLaunch {
+// A kernel launch as data (function, geometry, dynamic shared memory) for the
+// one-node launch graphs of runtime.cpp; err != cudaSuccess: not launchable.
+struct LaunchSpec {
     const void *func;
     int grid, block;
     size_t smem;
     cudaError_t err;
 };
+using FusedLaunch = LaunchSpec;
+// TMA bulk-copy variant of the fused kernel
 FusedLaunch fused_tma_launch(uint32_t nitems, int device);
+// pack_seal (register, geometry g) or pack_seal_tma; seal_reduce
+LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int device);
+LaunchSpec seal_reduce_launch(const SealReduceArgs &a);
 #ifndef VP_FUSED_TMA_DEFAULT
 #define VP_FUSED_TMA_DEFAULT 0
 #endif
