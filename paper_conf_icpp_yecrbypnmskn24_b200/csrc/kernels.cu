@@ -1150,6 +1150,24 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
     return l;
 }
 
+LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms) {
+    LaunchSpec l{};
+    if (tma) {
+        static std::atomic<uint64_t> opted{0};
+        const int sms = sm_count(device);
+        l.func = (const void *)install_verify_tma_kernel;
+        l.err = opt_in_smem(install_verify_tma_kernel, kTmaSmem, device, opted);
+        l.grid = grid_for(a.nitems, kTmaWarps, max_sms > 0 && max_sms < sms ? max_sms : sms, 2);
+        l.block = kTmaWarps * 32;
+        l.smem = kTmaSmem;
+    } else {
+        l.func = (const void *)install_verify_kernel;
+        l.grid = g.grid;
+        l.block = g.block;
+    }
+    return l;
+}
+
 LaunchSpec seal_reduce_launch(const SealReduceArgs &a) {
     LaunchSpec l{};
     l.func = (const void *)seal_reduce_kernel;

@@ -273,6 +273,47 @@ static void channel_close(Channel *ch) {
     delete ch;
 }
 
+cudaError_t OneNodeGraph::launch(const cudaKernelNodeParams &kp, cudaStream_t st) {
+    cudaError_t e;
+    if (x && func != kp.func) destroy();
+    if (!x) {
+        if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
+        if ((e = cudaGraphAddKernelNode(&n, g, nullptr, 0, &kp)) != cudaSuccess) return e;
+        if ((e = cudaGraphInstantiate(&x, g, 0)) != cudaSuccess) return e;
+        func = kp.func;
+    } else if ((e = cudaGraphExecKernelNodeSetParams(x, n, &kp)) != cudaSuccess) {
+        return e;
+    }
+    return cudaGraphLaunch(x, st);
+}
+
+void OneNodeGraph::destroy() {
+    if (x) cudaGraphExecDestroy(x);
+    if (g) cudaGraphDestroy(g);
+    x = nullptr;
+    g = nullptr;
+    n = nullptr;
+    func = nullptr;
+}
+
+static const bool g_no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));  // direct launches
+
+// A LaunchSpec with one by-value argument struct, through a one-node graph
+// (or directly with VIPER_NO_GRAPH=1).
+template <typename Args>
+static cudaError_t launch_spec(OneNodeGraph &og, const LaunchSpec &l, const Args &a, cudaStream_t st) {
+    if (l.err != cudaSuccess) return l.err;
+    void *args[] = {(void *)&a};
+    if (g_no_graph) return cudaLaunchKernel(l.func, dim3(l.grid), dim3(l.block), args, l.smem, st);
+    cudaKernelNodeParams kp{};
+    kp.func = (void *)l.func;
+    kp.gridDim = dim3(l.grid);
+    kp.blockDim = dim3(l.block);
+    kp.sharedMemBytes = (unsigned)l.smem;
+    kp.kernelParams = args;
+    return og.launch(kp, st);
+}
+
 // --------------------------------------------------------------- install path
 void fire_callback(viper_model *c, uint64_t v, viper_status st) {
     void (*cb)(uint64_t, viper_status, void *);
@@ -353,8 +394,8 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     const bool tma = direct && complete && !(c->cfg.flags & VIPER_FLAG_NO_TMA) &&
                      ((c->cfg.flags & VIPER_FLAG_TMA) || c->man.s_packed <= (1ull << 30));
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
-    if (tma) CUDA_TRY(launch_install_tma(pi.a, st, c->device, c->cfg.install_sms));
-    else CUDA_TRY(launch_install(pi.a, c->geo, st, pdl && !timing));
+    if (pdl && !timing && !tma) CUDA_TRY(launch_install(pi.a, c->geo, st, true));  // PDL: a plain stream launch
+    else CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms), pi.a, st));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
         c->timing_pending = true;
@@ -522,47 +563,6 @@ viper_status wait_install_done(viper_model *c, uint64_t v, cudaStream_t st) {
 int64_t g_trace[16];  // debug: host timestamps of the last publish (viper_debug_trace)
 static const bool g_trace_on = getenv("VIPER_TRACE") != nullptr;  // tools/trace_publish.py sets it
 #define TRACE(i) (g_trace_on ? (void)(g_trace[i] = now_ns()) : (void)0)
-
-cudaError_t OneNodeGraph::launch(const cudaKernelNodeParams &kp, cudaStream_t st) {
-    cudaError_t e;
-    if (x && func != kp.func) destroy();
-    if (!x) {
-        if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
-        if ((e = cudaGraphAddKernelNode(&n, g, nullptr, 0, &kp)) != cudaSuccess) return e;
-        if ((e = cudaGraphInstantiate(&x, g, 0)) != cudaSuccess) return e;
-        func = kp.func;
-    } else if ((e = cudaGraphExecKernelNodeSetParams(x, n, &kp)) != cudaSuccess) {
-        return e;
-    }
-    return cudaGraphLaunch(x, st);
-}
-
-void OneNodeGraph::destroy() {
-    if (x) cudaGraphExecDestroy(x);
-    if (g) cudaGraphDestroy(g);
-    x = nullptr;
-    g = nullptr;
-    n = nullptr;
-    func = nullptr;
-}
-
-static const bool g_no_graph = getenv("VIPER_NO_GRAPH") && atoi(getenv("VIPER_NO_GRAPH"));  // direct launches
-
-// A LaunchSpec with one by-value argument struct, through a one-node graph
-// (or directly with VIPER_NO_GRAPH=1).
-template <typename Args>
-static cudaError_t launch_spec(OneNodeGraph &og, const LaunchSpec &l, const Args &a, cudaStream_t st) {
-    if (l.err != cudaSuccess) return l.err;
-    void *args[] = {(void *)&a};
-    if (g_no_graph) return cudaLaunchKernel(l.func, dim3(l.grid), dim3(l.block), args, l.smem, st);
-    cudaKernelNodeParams kp{};
-    kp.func = (void *)l.func;
-    kp.gridDim = dim3(l.grid);
-    kp.blockDim = dim3(l.block);
-    kp.sharedMemBytes = (unsigned)l.smem;
-    kp.kernelParams = args;
-    return og.launch(kp, st);
-}
 
 // The fused kernel through its one-node graph: measured cheaper on the host
 // than a direct launch (profiles/r01/launchcal.log).
@@ -889,6 +889,7 @@ static void free_model(viper_model *m) {
     m->g_fused.destroy();
     m->g_pack.destroy();
     m->g_seal.destroy();
+    m->g_inst.destroy();
     if (m->side) cudaStreamDestroy(m->side);
     if (m->ustream) cudaStreamDestroy(m->ustream);
     delete m;

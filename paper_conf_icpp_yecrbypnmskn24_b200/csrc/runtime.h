@@ -148,6 +148,7 @@ struct viper_model {
     bool timing_pending = false;
     bool last_fused = false;                         // last publish used publish_fused_kernel
     vp::OneNodeGraph g_fused, g_pack, g_seal;        // per-publish launches through one-node graphs
+    vp::OneNodeGraph g_inst;                         // consumer: installs not PDL-chained (install_mu held)
     cudaStream_t side = nullptr;                     // DRAM-tier D2H stream
     uint8_t *h_stage[2] = {nullptr, nullptr};        // DRAM tier (pinned)
     vp::ISeal *h_iseal[2] = {nullptr, nullptr};

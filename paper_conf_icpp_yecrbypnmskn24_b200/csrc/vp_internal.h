@@ -153,6 +153,8 @@ FusedLaunch fused_tma_launch(uint32_t nitems, int device);
 // pack_seal (register, geometry g) or pack_seal_tma; seal_reduce
 LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int device);
 LaunchSpec seal_reduce_launch(const SealReduceArgs &a);
+// install_verify (register, geometry g, not PDL-chained) or install_verify_tma
+LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms);
 #ifndef VP_FUSED_TMA_DEFAULT
 #define VP_FUSED_TMA_DEFAULT 0
 #endif
