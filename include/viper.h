@@ -305,6 +305,13 @@ viper_status viper_debug_proto_publish(void *h, uint64_t v);
 viper_status viper_debug_proto_install(void *h, int32_t cidx, uint64_t *installed, uint64_t *torn_snapshot);
 viper_status viper_debug_proto_read(void *h, int32_t cidx, uint64_t *version, uint64_t *torn);
 
+/* Test hook: the Transfer Selector's decision (VIPER_TIER_AUTO, selector.h)
+ * on `world` gathered 288-byte records {u32 magic 0x56495452, i32 tier,
+ * i32 nreach, i32 pad, char pci[16], char reach[16][16]}, as every rank of the
+ * cross-process bootstrap computes it.  *out = the tier in use.  Host only. */
+viper_status viper_debug_resolve_tier(const void *records, int32_t world, int32_t producer_rank,
+                                      int32_t nproducers, int32_t fanout, int32_t requested, int32_t *out);
+
 /* Tear down (joins the update thread, frees library-owned memory). */
 viper_status viper_unregister(viper_model *m);
 

@@ -18,6 +18,7 @@
 
 #include "protocol.h"
 #include "runtime.h"
+#include "selector.h"
 
 using namespace vp;
 
@@ -160,6 +161,16 @@ viper_status viper_debug_proto_read(void *h, int32_t cidx, uint64_t *version, ui
     release_slot(r, slot);
     *version = v;
     *torn = bad;
+    return VIPER_OK;
+}
+
+// Transfer Selector (selector.h) on synthetic gathered records.
+viper_status viper_debug_resolve_tier(const void *records, int32_t world, int32_t producer_rank,
+                                      int32_t nproducers, int32_t fanout, int32_t requested, int32_t *out) {
+    const int M = nproducers > 1 ? nproducers : 1;
+    if (!records || !out || world < 1 || producer_rank < 0 || producer_rank + M > world)
+        return set_error(VIPER_E_INVAL, "bad arguments");
+    *out = resolve_tier((const TierRec *)records, world, producer_rank, M, fanout, requested);
     return VIPER_OK;
 }
 

@@ -28,24 +28,13 @@
 
 #include "protocol.h"
 #include "runtime.h"
+#include "selector.h"
 
 namespace vp {
 
 namespace {
 
 constexpr uint32_t kPeerMagic = 0x56495052u;  // "VIPR"
-constexpr uint32_t kTierMagic = 0x56495452u;  // "VITR"
-constexpr int kMaxReach = 16;
-
-// Transfer Selector round (the first bootstrap allgather, every rank): the
-// tier asked for and the GPUs this rank's GPU can reach (itself included), as
-// PCI bus ids, so that every rank resolves VIPER_TIER_AUTO from the same data.
-struct TierRec {
-    uint32_t magic;
-    int32_t tier, nreach, pad;
-    char pci[16];
-    char reach[kMaxReach][16];
-};
 
 struct PeerRec {
     uint32_t magic;
@@ -244,23 +233,8 @@ int32_t select_tier_xproc(const viper_model *m, const viper_bootstrap *bs, int M
     }
     std::vector<TierRec> all(bs->world);
     *comm_ok = bs->allgather(&me, all.data(), sizeof(TierRec), bs->user) == 0;
-    if (!*comm_ok || m->cfg.tier != VIPER_TIER_AUTO) return m->cfg.tier;
-    auto producer = [&](int r) { return r >= bs->producer_rank && r < bs->producer_rank + M; };
-    auto reaches = [&](int a, int b) {  // rank a's GPU can read rank b's GPU memory
-        if (all[a].magic != kTierMagic || all[b].magic != kTierMagic) return true;
-        for (int k = 0; k < all[a].nreach && k < kMaxReach; k++)
-            if (strncmp(all[a].reach[k], all[b].pci, 16) == 0) return true;
-        return false;
-    };
-    // consumers pull from the producers, and with chain / scatter-allgather
-    // fan-out also from each other
-    const bool peers = m->cfg.fanout == VIPER_FANOUT_CHAIN || m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER;
-    for (int c = 0; c < bs->world; c++) {
-        if (producer(c)) continue;
-        for (int r = 0; r < bs->world; r++)
-            if (r != c && (producer(r) || peers) && !reaches(c, r)) return VIPER_TIER_DRAM;
-    }
-    return VIPER_TIER_GPU;
+    if (!*comm_ok) return m->cfg.tier;
+    return resolve_tier(all.data(), bs->world, bs->producer_rank, M, m->cfg.fanout, m->cfg.tier);
 }
 
 }  // namespace

@@ -83,7 +83,8 @@ EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_ac
            "viper_wait_installed", "viper_get_stats", "viper_layout", "viper_debug_buffers", "viper_debug_fault_next", "viper_unregister",
            "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version",
            "viper_debug_proto_create", "viper_debug_proto_open", "viper_debug_proto_close",
-           "viper_debug_proto_publish", "viper_debug_proto_install", "viper_debug_proto_read"]
+           "viper_debug_proto_publish", "viper_debug_proto_install", "viper_debug_proto_read",
+           "viper_debug_resolve_tier"]
 
 _lib = None
 _lock = threading.Lock()
@@ -130,6 +131,8 @@ def lib() -> C.CDLL:
             L.viper_debug_proto_install.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_uint64),
                                                     C.POINTER(C.c_uint64)]
             L.viper_debug_proto_read.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]
+            L.viper_debug_resolve_tier.argtypes = [C.c_void_p, C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_int32,
+                                                   C.POINTER(C.c_int32)]
             L.viper_restore.argtypes = [C.c_char_p, C.POINTER(viper_tensor), C.c_int32, C.c_int32, C.c_void_p,
                                         C.POINTER(C.c_uint64)]
             L.viper_strerror.argtypes = [C.c_int32]
