@@ -277,9 +277,12 @@ cudaError_t OneNodeGraph::launch(const cudaKernelNodeParams &kp, cudaStream_t st
     cudaError_t e;
     if (x && func != kp.func) destroy();
     if (!x) {
-        if ((e = cudaGraphCreate(&g, 0)) != cudaSuccess) return e;
-        if ((e = cudaGraphAddKernelNode(&n, g, nullptr, 0, &kp)) != cudaSuccess) return e;
-        if ((e = cudaGraphInstantiate(&x, g, 0)) != cudaSuccess) return e;
+        if ((e = cudaGraphCreate(&g, 0)) == cudaSuccess && (e = cudaGraphAddKernelNode(&n, g, nullptr, 0, &kp)) == cudaSuccess)
+            e = cudaGraphInstantiate(&x, g, 0);
+        if (e != cudaSuccess) {
+            destroy();  // nothing half-built is kept; the next launch starts over
+            return e;
+        }
         func = kp.func;
     } else if ((e = cudaGraphExecKernelNodeSetParams(x, n, &kp)) != cudaSuccess) {
         return e;
