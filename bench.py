@@ -43,6 +43,9 @@ sys.path.insert(0, ROOT)
 
 HBM_NOMINAL_GBS = 7700.0  # B200 HGX HBM3e nominal (B200_PROFILING.md), context beside the measured copy peak
 METRIC = "model-update latency (ms) and GB/s vs NVLink/HBM roofline at 1->1/3/7 GPUs"
+# "dtype" is the arithmetic the path computes in: bytes moved as 128-bit words,
+# sealed with u32 word checksums summed mod 2^64 (R16); the model's
+# own element type, never interpreted, is reported as "model_dtype".
 
 
 def load_peaks():
@@ -714,7 +717,7 @@ def xproc_arm(args):
         out = {
             "metric": METRIC, "value": round(lat_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(lat_ms, 6), "higher_is_better": False, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+            "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
             "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
             "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers "
                                    f"{'sharing one GPU (code path only, no NVLink)' if over else 'over NVLink'} "
@@ -796,7 +799,7 @@ def gpu_arm(args):
     out = {
         "metric": METRIC, "value": round(mean_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(mean_ms, 6), "higher_is_better": False,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+        "scaling": "weak", "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
         "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
         "config": {"workload": f"{name}: 1 producer -> 1 consumer, 1-GPU loopback "
                                f"(BASELINE.json configs[{CONFIG_INDEX[name]}]"
@@ -926,7 +929,7 @@ def reference_arm(args):
     v = statistics.mean(res)
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "ms", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(v, 4), "higher_is_better": False,
-           "scaling": "weak", "vs_baseline": None, "dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+           "scaling": "weak", "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
            "data": "synthetic (VGEN)", "config": {"workload": f"{name}: 1 producer -> 1 consumer, the oracle on host cores "
                                                      f"(BASELINE.json configs[{CONFIG_INDEX[name]}])"},
            "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
