@@ -604,6 +604,34 @@ __device__ __forceinline__ void bulk_g2s(void *smem, const void *gmem, uint32_t 
                  : "memory");
 }
 
+#ifndef VP_TMA_HINTS
+#define VP_TMA_HINTS 1  // 0: compile the L2 hints out (A/B, profiles/r01/tma_l2_hint_ab.log)
+#endif
+// L2 policy for data read exactly once (the pack's parameter tensors, the
+// install's snapshot): evict it first, so it does not push out data that is
+// read again soon (the snapshot the install or the D2H reads next).
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
+// pol == 0: no hint (models larger than L2 gain nothing from it and lose a little)
+__device__ __forceinline__ void bulk_g2s_once(void *smem, const void *gmem, uint32_t bytes, uint64_t *bar,
+                                              uint64_t pol) {
+#if VP_TMA_HINTS
+    if (pol) {
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], "
+            "%4;" ::"r"(smem_u32(smem)),
+            "l"(gmem), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+            : "memory");
+        return;
+    }
+#endif
+    bulk_g2s(smem, gmem, bytes, bar);
+}
+
 __device__ __forceinline__ void bulk_s2g(void *gmem, const void *smem, uint32_t bytes) {
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gmem), "r"(smem_u32(smem)),
                  "r"(bytes)
@@ -629,6 +657,7 @@ __device__ __forceinline__ uint32_t tma_body(const Item &it) {
 __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const PackArgs a) {
     extern __shared__ __align__(128) uint8_t tma_smem[];
     const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint64_t pol = a.l2_once ? l2_evict_first_policy() : 0;  // parameter tensors: read once
     uint8_t *stage = tma_smem + wib * (kTmaStages * kTmaStage);
     uint64_t *bar = reinterpret_cast<uint64_t *>(tma_smem + kTmaWarps * kTmaStages * kTmaStage) + wib * kTmaStages;
     if (lane == 0) {
@@ -661,7 +690,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const 
         if (!next_piece(ld, it, bytes)) break;
         if (lane == 0) {
             mbar_expect_tx(bar + s, bytes);
-            bulk_g2s(stage + s * kTmaStage, (const uint8_t *)it.ptr + ld.off, bytes, bar + s);
+            bulk_g2s_once(stage + s * kTmaStage, (const uint8_t *)it.ptr + ld.off, bytes, bar + s, pol);
         }
         ld.off += bytes;
         issued++;
@@ -693,7 +722,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const 
                 if (lane == 0) {
                     bulk_wait_read<0>();
                     mbar_expect_tx(bar + s, nbytes);
-                    bulk_g2s(stage + s * kTmaStage, (const uint8_t *)nit.ptr + ld.off, nbytes, bar + s);
+                    bulk_g2s_once(stage + s * kTmaStage, (const uint8_t *)nit.ptr + ld.off, nbytes, bar + s, pol);
                 }
                 ld.off += nbytes;
                 issued++;
@@ -722,6 +751,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) pack_seal_tma_kernel(const 
 __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(const InstallArgs a) {
     extern __shared__ __align__(128) uint8_t tma_smem[];
     const uint32_t lane = threadIdx.x & 31u, wib = threadIdx.x >> 5;
+    const uint64_t pol = a.l2_once ? l2_evict_first_policy() : 0;  // the snapshot: read once
     uint8_t *stage = tma_smem + wib * (kTmaStages * kTmaStage);
     uint64_t *bar = reinterpret_cast<uint64_t *>(tma_smem + kTmaWarps * kTmaStages * kTmaStage) + wib * kTmaStages;
     if (lane == 0) {
@@ -754,7 +784,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
         if (!next_piece(ld, it, bytes)) break;
         if (lane == 0) {
             mbar_expect_tx(bar + s, bytes);
-            bulk_g2s(stage + s * kTmaStage, a.packed + it.packed_off + ld.off, bytes, bar + s);
+            bulk_g2s_once(stage + s * kTmaStage, a.packed + it.packed_off + ld.off, bytes, bar + s, pol);
         }
         ld.off += bytes;
     }
@@ -800,7 +830,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
                 if (lane == 0) {
                     bulk_wait_read<0>();
                     mbar_expect_tx(bar + s, nbytes);
-                    bulk_g2s(stage + s * kTmaStage, a.packed + nit.packed_off + ld.off, nbytes, bar + s);
+                    bulk_g2s_once(stage + s * kTmaStage, a.packed + nit.packed_off + ld.off, nbytes, bar + s, pol);
                 }
                 ld.off += nbytes;
             }

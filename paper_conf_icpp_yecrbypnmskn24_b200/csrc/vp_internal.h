@@ -51,6 +51,8 @@ struct PackArgs {
     uint64_t version;
     uint32_t sys_release;       // release the ready flags at system scope (consumers
                                 // on other GPUs pipeline behind this pack)
+    uint32_t l2_once;           // TMA variant: load the tensors with an L2 evict-first hint
+                                // (set when the snapshot fits in L2, so it stays there)
 };
 
 struct SealReduceArgs {
@@ -98,6 +100,7 @@ struct InstallArgs {
     const uint8_t *const *sa_src;                // [sa_n] peers' staging (device-mapped)
     const ISeal *const *sa_isrc;                 // [sa_n] peers' staging seals
     const volatile uint64_t *const *sa_owner_pin;  // [sa_n] peers' pin words (host-mapped)
+    uint32_t l2_once;           // TMA variant: load the snapshot with an L2 evict-first hint
 };
 
 // SYNC in-process publish (K2+K6 fused): each warp packs its item,
