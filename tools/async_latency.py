@@ -18,13 +18,14 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="resnet50")
 ap.add_argument("--steps", type=int, default=20)
 ap.add_argument("--gap-ms", type=float, default=2.0, help="idle time between updates (the update thread sleeps)")
+ap.add_argument("--tier", type=int, default=0, help="0 GPU, 1 DRAM")
 a = ap.parse_args()
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
-c = V.Model("al", V.CONSUMER, ct)
-p = V.Model("al", V.PRODUCER, pt, mode=V.ASYNC)
+c = V.Model("al", V.CONSUMER, ct, tier=a.tier)
+p = V.Model("al", V.PRODUCER, pt, mode=V.ASYNC, tier=a.tier)
 stall, done, pick, inst = [], [], [], []
 for v in range(1, a.steps + 4):
     G.fill_model(pt, specs, seed, v)
@@ -45,5 +46,5 @@ for v in range(1, a.steps + 4):
 c.close()
 p.close()
 med = statistics.median
-print(f"{a.config} ASYNC: publish returns {med(stall):.1f} us | pickup {med(pick):.1f} us | "
+print(f"{a.config} tier={a.tier} ASYNC: publish returns {med(stall):.1f} us | pickup {med(pick):.1f} us | "
       f"install (launch->done) {med(inst):.1f} us | publish -> installed {med(done):.1f} us")
