@@ -275,3 +275,32 @@ def random_specs(rng: np.random.Generator, n: int, max_bytes: int = 67, dtypes=(
         ne = int(rng.integers(0, max_bytes // es + 1))
         out.append((f"t{i}", dt, (ne,)))
     return out
+
+
+# --------------------------------------------------------------------------
+# Verification content (golden seals)
+# --------------------------------------------------------------------------
+# The VGEN version whose packed chunk checksums tools/make_golden_seals.py
+# wrote into tests/golden/seals/<model>.txt with the ORACLE.  Multi-GPU bench
+# runs and GPU tests publish this content as their last version and compare
+# every consumer's installed seals against that file.
+VCHECK = 7
+
+
+def golden_seals(name: str):
+    """(header dict, list of chunk cks ints) from tests/golden/seals/<name>.txt
+    (values written by the oracle; this only parses the file), or None."""
+    import os
+    path = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests", "golden", "seals",
+                        f"{name}.txt")
+    if not os.path.exists(path):
+        return None
+    with open(path) as f:
+        head = f.readline().lstrip("#").split()
+        hdr = {k: v for k, v in (kv.split("=", 1) for kv in head)}
+        cks = [int(line, 16) for line in f if line.strip()]
+    for k in ("content_version", "chunk_bytes", "s_packed", "nchunks"):
+        hdr[k] = int(hdr[k])
+    if hdr["nchunks"] != len(cks) or hdr["content_version"] != VCHECK:
+        raise ValueError(f"{path}: malformed golden seal file")
+    return hdr, cks
