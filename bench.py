@@ -223,6 +223,78 @@ def run_update_bench(V, G, synth, name, steps, warmup, flush_buf, mode=None, tie
             "s_packed": s_packed, "nchunks": nchunks, "bytes": synth.model_bytes(name), "tensors": len(specs)}
 
 
+def run_back_to_back(V, G, synth, name, steps, warmup):
+    """Steady state: K SYNC publishes issued back to back with
+    nothing in between (no L2 flush, no optimizer write), one CUDA-event window
+    around all K on the publishing stream: every update pays the deferred L2
+    write-back of the one before it.  ms per update."""
+    import torch
+    specs = synth.model_specs(name)
+    prod_t, cons_t = G.alloc_model(specs), G.alloc_model(specs)
+    G.fill_model(prod_t, specs, synth.SEEDS[name], 1)
+    mname = f"b2b-{name}-{os.getpid()}-{time.monotonic_ns()}"
+    cons = V.Model(mname, V.CONSUMER, cons_t)
+    prod = V.Model(mname, V.PRODUCER, prod_t)
+    st = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    try:
+        for v in range(1, warmup + 1):
+            prod.publish(v, stream=st)
+        torch.cuda.synchronize()
+        e0.record(st)
+        for v in range(warmup + 1, warmup + steps + 1):
+            prod.publish(v, stream=st)
+        e1.record(st)
+        e1.synchronize()
+        view = cons.acquire_latest()
+        ok = view.version == warmup + steps and all(
+            torch.equal(g.view(torch.uint8), p.view(torch.uint8)) for g, p in zip(view.tensors(cons_t), prod_t))
+        cons.release(view)
+    finally:
+        cons.close()
+        prod.close()
+    return e0.elapsed_time(e1) / steps, ok
+
+
+def golden_check_local(V, G, synth, name):
+    """The N = 1 headline config's bit-exact evidence against the oracle: publish
+    VGEN(seed, synth.VCHECK) and compare the producer's chunk seals and the
+    consumer's installed-slot seals (viper_view_seals) with the oracle-written
+    tests/golden/seals/<name>.txt, plus every byte of the slot with VGEN."""
+    import numpy as np
+    import torch
+    specs = synth.model_specs(name)
+    gold = synth.golden_seals(name)
+    prod_t, cons_t = G.alloc_model(specs), G.alloc_model(specs)
+    G.fill_model(prod_t, specs, synth.SEEDS[name], synth.VCHECK)
+    mname = f"gold-{name}-{os.getpid()}-{time.monotonic_ns()}"
+    cons = V.Model(mname, V.CONSUMER, cons_t)
+    prod = V.Model(mname, V.PRODUCER, prod_t)
+    try:
+        prod.publish(1)
+        _, sp, n = prod.debug_buffers()
+        like = torch.empty(4 * n, dtype=torch.int32, device="cuda")
+        pseals = V._from_ptr(sp, like).view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2)
+        view = cons.acquire_latest()
+        buf = torch.empty(16 * n, dtype=torch.uint8, device="cuda")
+        cons.view_seals(view, buf)
+        torch.cuda.synchronize()
+        cseals = buf.view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2)
+        exp = G.alloc_model(specs)
+        G.fill_model(exp, specs, synth.SEEDS[name], synth.VCHECK)
+        bytes_ok = all(torch.equal(g.view(torch.uint8), e.view(torch.uint8)) for g, e in zip(view.tensors(cons_t), exp))
+        cons.release(view)
+    finally:
+        cons.close()
+        prod.close()
+    g = np.array(gold[1], dtype=np.uint64) if gold else None
+    return {"chunks": n, "producer_seals_ok": bool(g is not None and np.array_equal(pseals[:, 1], g)),
+            "consumer_seals_ok": bool(g is not None and np.array_equal(cseals[:, 1], g) and (cseals[:, 0] == 1).all()),
+            "bytes_ok": bool(bytes_ok),
+            "how": "VGEN(seed, synth.VCHECK) published; every chunk seal of the snapshot and of the consumer's "
+                   "installed slot (viper_view_seals) == the oracle's tests/golden/seals file; every slot byte == VGEN"}
+
+
 def run_e2e(V, G, synth, name, steps, warmup, flush_buf):
     """Same update through the public API with HOST buffers: the trainer's
     parameters live in one flat device buffer (tensor views at 256-B aligned
@@ -471,47 +543,92 @@ def cpu_model():
 
 class OracleUpdates:
     """The oracle (plain C, single thread, as it stands) set up once for one
-    config: a producer + 1 consumer and two pre-generated versions."""
+    config: a producer + `ncons` consumers and two pre-generated versions.
+    `subset`: only these tensor indices (the P-thread baseline gives each
+    thread a disjoint subset, its own oracle channel)."""
 
-    def __init__(self, synth, name):
+    def __init__(self, synth, name, ncons=1, subset=None):
         from oracle import transfer as T
         self.T, self.name = T, name
         specs = synth.model_specs(name)
         seed = synth.SEEDS[name]
-        nb = [synth.nbytes_of(s) for s in specs]
-        self.versions = [[synth.vgen_numpy(seed, v, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
+        idx = list(range(len(specs))) if subset is None else list(subset)
+        nb = [synth.nbytes_of(specs[i]) for i in idx]
+        self.versions = [[synth.vgen_numpy(seed, v, i, specs[i][1], synth.nelem_of(specs[i])) for i in idx]
                          for v in (1, 2)]
-        self.c = self.T.Consumer(nb)
-        self.p = self.T.Producer(nb, [self.c])
+        self.cs = [self.T.Consumer(nb) for _ in range(ncons)]
+        self.p = self.T.Producer(nb, self.cs)
         self.v = 0
+
+    def one(self):
+        self.v += 1
+        st = self.p.publish(self.v, self.versions[self.v % 2])
+        assert st == self.T.OK
 
     def run(self, budget_s, max_updates=100000):
         """Updates until the budget is spent; ms per update."""
         times = []
         t_start = time.perf_counter()
         while time.perf_counter() - t_start < budget_s and len(times) < max_updates:
-            self.v += 1
             t0 = time.perf_counter()
-            st = self.p.publish(self.v, self.versions[self.v % 2])
+            self.one()
             times.append((time.perf_counter() - t0) * 1e3)
-            assert st == self.T.OK
         return times
 
     def close(self):
         self.p.close()
-        self.c.close()
+        for c in self.cs:
+            c.close()
+
+
+def oracle_parallel(synth, name, nthreads, budget_s, max_updates=100000):
+    """P-thread oracle baseline: the model's tensors split into
+    P disjoint subsets of about equal bytes, each its own oracle channel (plain
+    C, single-threaded, unchanged) driven by its own thread; one update = every
+    thread updating its subset (the ctypes calls release the GIL).  ms per
+    whole-model update."""
+    specs = synth.model_specs(name)
+    order = sorted(range(len(specs)), key=lambda i: -synth.nbytes_of(specs[i]))
+    groups, load = [[] for _ in range(nthreads)], [0] * nthreads
+    for i in order:  # greedy: largest tensor to the lightest group
+        k = load.index(min(load))
+        groups[k].append(i)
+        load[k] += synth.nbytes_of(specs[i])
+    groups = [sorted(g) for g in groups if g]
+    parts = [OracleUpdates(synth, name, subset=g) for g in groups]
+    times = []
+    try:
+        t_start = time.perf_counter()
+        while time.perf_counter() - t_start < budget_s and len(times) < max_updates:
+            ths = [threading.Thread(target=o.one) for o in parts]
+            t0 = time.perf_counter()
+            for th in ths:
+                th.start()
+            for th in ths:
+                th.join()
+            times.append((time.perf_counter() - t0) * 1e3)
+    finally:
+        for o in parts:
+            o.close()
+    return times, len(parts)
 
 
 def cpu_baseline(synth, name, budget_s=10.0, max_updates=100000):
     """The oracle timed on this host's cores on a bounded sample: repeated
-    updates of the same config."""
+    updates of the same config, on 1 thread (the value) and on P threads
+    (P = the cores this process may use)."""
     o = OracleUpdates(synth, name)
     try:
         times = o.run(budget_s, max_updates)
     finally:
         o.close()
-    return {"value": statistics.mean(times), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
-            "sample": f"{len(times)} oracle updates of {name} (pack+seal+deliver+verify+install+swap, 1 consumer)"}
+    cpu = cpu_model()
+    ptimes, p = oracle_parallel(synth, name, cpu["affinity_cores"], budget_s, max_updates)
+    return {"value": statistics.mean(times), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu,
+            "sample": f"{len(times)} oracle updates of {name} (pack+seal+deliver+verify+install+swap, 1 consumer)",
+            "p_threads": {"value": statistics.mean(ptimes), "unit": "ms", "cores": p, "kind": "oracle",
+                          "sample": f"{len(ptimes)} whole-model updates of {name}, the tensors split into {p} "
+                                    f"disjoint subsets of about equal bytes, one oracle channel and thread each"}}
 
 
 N_CONFIG = {2: "resnet50", 4: "vit_b16", 8: "gpt2_xl"}  # BASELINE.json configs[1..3]
@@ -616,49 +733,86 @@ def xproc_e2e(V, G, synth, name, rank, world, dev, group, fanout, flush_buf, ste
     return {"ms": statistics.mean(times) if times else 0.0, "h2d": flat.numel(), "d2h": 16 * nchunks, "ok": ok}
 
 
-def xproc_arm(args):
-    """N > 1: one process per GPU.  Rank 0 is the producer, ranks 1..N-1 the
-    consumers (1 -> N-1 fan-out over NVLink: direct for one consumer,
-    scatter-allgather for more; --fanout chain picks the pipelined chain).  Each step is one SYNC update: rank 0's
-    publish() returns once every consumer swapped.  value = mean update
-    latency (host clock of rank 0 from publish entry to the last consumer's
-    swap); consumers' install-kernel times (CUDA events) are
-    reported as the max over ranks.  An NCCL broadcast of the packed bytes is
-    timed beside it as the baseline."""
+FANOUTS = {"direct": 0, "chain": 1, "sa": 2, "nvls": 3, "push": 4, "ce": 101}  # include/viper.h VIPER_FANOUT_*
+FANOUT_NAMES = {0: "direct pull", 1: "pipelined chain", 2: "scatter-allgather", 3: "NVLS multicast",
+                4: "push (producer stores into peer staging)", 101: "copy engine (engine baseline)"}
+NVLINK_GBS = 900.0  # NVLink 5 per direction per GPU (north_star / B200_PROFILING.md)
+
+
+def verify_replicas(V, G, synth, m, name, rank, tensors, dev):
+    """Bit-exact evidence for one cross-process run, without the oracle at bench
+    time: the LAST published version carries VGEN(seed, synth.VCHECK), whose
+    chunk checksums tools/make_golden_seals.py wrote with the oracle into
+    tests/golden/seals/<name>.txt.  Each consumer computes the chunk seals of
+    its installed slot on its GPU (viper_view_seals) and compares EVERY chunk
+    with that file, then compares every byte of every tensor with VGEN
+    regenerated on its GPU; the producer compares its snapshot seals.  Returns
+    {"seals_ok", "bytes_ok", "chunks", "version"}."""
+    import numpy as np
+    import torch
+    gold = synth.golden_seals(name)
+    specs = synth.model_specs(name)
+    out = {"seals_ok": None, "bytes_ok": None, "chunks": 0, "version": 0}
+    if rank == 0:
+        _, sp, n = m.debug_buffers()
+        like = torch.empty(4 * n, dtype=torch.int32, device=f"cuda:{dev}")
+        seals = V._from_ptr(sp, like).view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2)
+        out["version"] = int(seals[0, 0]) if n else 0
+        if gold is not None:
+            out["seals_ok"] = bool(n == gold[0]["nchunks"] and all(int(seals[c, 1]) == gold[1][c] for c in range(n)))
+            out["chunks"] = n
+        return out
+    view = m.acquire_latest(timeout_us=30_000_000)
+    try:
+        n = m.stats()["nchunks"]
+        buf = torch.empty(max(16 * n, 16), dtype=torch.uint8, device=f"cuda:{dev}")
+        st = torch.cuda.current_stream()
+        m.view_seals(view, buf, stream=st)
+        st.synchronize()
+        got = buf.view(torch.int64).cpu().numpy().view(np.uint64).reshape(-1, 2)[:n]
+        out["version"] = int(view.version)
+        out["chunks"] = n
+        if gold is not None:
+            out["seals_ok"] = bool(n == gold[0]["nchunks"] and (got[:, 0] == view.version).all()
+                                   and all(int(got[c, 1]) == gold[1][c] for c in range(n)))
+        exp = G.alloc_model(specs, device=f"cuda:{dev}")
+        G.fill_model(exp, specs, synth.SEEDS[name], synth.VCHECK)
+        out["bytes_ok"] = bool(all(torch.equal(g.view(torch.uint8), e.view(torch.uint8))
+                                   for g, e in zip(view.tensors(tensors), exp)))
+        del exp
+    finally:
+        m.release(view)
+    return out
+
+
+def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, steps, warmup):
+    """One fan-out, SYNC updates.  Per step (untimed): VGEN(v) into the
+    producer's tensors, an L2 flush on every rank, barrier.  Timed: CUDA events
+    on rank 0's stream around publish(v), which returns only once every
+    consumer's install kernel swapped its version word (so the window holds the
+    whole pack -> NVLink -> install pipeline); host clock beside it.  Consumers
+    report their install kernel's CUDA-event time (VIPER_FLAG_TIMING).  Then the
+    verification version (verify_replicas).  Returns this rank's dict, or
+    {"unsupported": why} on every rank when registration says so (NVLS without
+    multicast, ...)."""
     import torch
     import torch.distributed as dist
-    import synth
-    from synth import gpu as G
-    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
-    rank, world, local = dist_env()
-    ndev = torch.cuda.device_count()
-    dev = local % ndev
-    torch.cuda.set_device(dev)
-    over = ndev < world  # more ranks than GPUs (code-path testing on a 1-GPU box): no NCCL
-    if over:
-        dist.init_process_group("gloo")
-    else:
-        dist.init_process_group("cpu:gloo,cuda:nccl", device_id=torch.device("cuda", dev))
-    name = args.config if args.config_explicit else N_CONFIG.get(world, "resnet50")
     specs = synth.model_specs(name)
     seed = synth.SEEDS[name]
     tensors = G.alloc_model(specs)
-    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device="cuda")
-    gloo = dist.new_group(backend="gloo")
     bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
-    # auto: scatter-allgather for 1 -> N > 1 over NVLink; direct pulls when the
-    # ranks share GPUs (oversubscribed code-path runs: peers time-slice one GPU,
-    # so waiting on a peer's staged copy only serialises the installs)
-    fanout = {"direct": V.FANOUT_DIRECT, "chain": V.FANOUT_CHAIN, "sa": V.FANOUT_SCATTER_ALLGATHER}.get(
-        args.fanout, V.FANOUT_SCATTER_ALLGATHER if world > 2 and not over else V.FANOUT_DIRECT)
-    fanout_name = {V.FANOUT_DIRECT: "direct pull", V.FANOUT_CHAIN: "pipelined chain",
-                   V.FANOUT_SCATTER_ALLGATHER: "scatter-allgather"}[fanout]
-    role = V.PRODUCER if rank == 0 else V.CONSUMER
-    m = V.Model(f"bench-x-{name}", role, tensors, fanout=fanout, flags=V.FLAG_TIMING if rank else 0,
-                device=dev, bootstrap=bs)
-    lat, inst = [], []
-    with ClockSampler(dev) as clk:
-        for i in range(args.warmup + args.steps):
+    try:
+        m = V.Model(f"bench-x-{name}-{fanout}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors, fanout=fanout,
+                    flags=V.FLAG_TIMING if rank else 0, device=dev, bootstrap=bs)
+    except V.ViperError as e:
+        del tensors
+        torch.cuda.empty_cache()
+        return {"unsupported": f"{e.name}: {e.detail}"[:300]}
+    st = torch.cuda.current_stream()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    lat, host, inst = [], [], []
+    try:
+        for i in range(warmup + steps):
             v = i + 1
             if rank == 0:
                 G.fill_model(tensors, specs, seed, v)
@@ -666,28 +820,239 @@ def xproc_arm(args):
             torch.cuda.synchronize()
             dist.barrier(group=gloo)
             if rank == 0:
+                ev0.record(st)
                 t0 = time.perf_counter()
-                m.publish(v)
-                lat.append((time.perf_counter() - t0) * 1e3)
+                m.publish(v, stream=st)
+                t1 = time.perf_counter()
+                ev1.record(st)
+                ev1.synchronize()
+                if i >= warmup:
+                    lat.append(ev0.elapsed_time(ev1))
+                    host.append((t1 - t0) * 1e3)
             dist.barrier(group=gloo)
-            if rank != 0:
+            if rank != 0 and i >= warmup:
                 inst.append(m.stats()["t_install_dev_us"])
-    ok = 1
-    if rank != 0:
-        view = m.acquire_latest()
-        exp = [synth.vgen_bytes_range(seed, view.version, t, s[1], 0, min(4096, synth.nbytes_of(s)))
-               for t, s in enumerate(specs)]
-        got = view.tensors(tensors)
-        import numpy as np
-        for g, e in zip(got, exp):
-            b_ = g.contiguous().view(torch.uint8).reshape(-1)[:e.size].cpu().numpy()
-            ok &= int(np.array_equal(b_, e))
-        ok &= int(view.version == args.warmup + args.steps)
-        m.release(view)
-    # NCCL broadcast baseline of the same bytes (timed on the device, max over ranks)
+        # verification version: the golden content
+        if rank == 0:
+            G.fill_model(tensors, specs, seed, synth.VCHECK)
+            torch.cuda.synchronize()
+        dist.barrier(group=gloo)
+        if rank == 0:
+            m.publish(warmup + steps + 1, stream=st)
+            st.synchronize()
+        dist.barrier(group=gloo)
+        ver = verify_replicas(V, G, synth, m, name, rank, tensors, dev)
+        ver["version_ok"] = ver["version"] == warmup + steps + 1
+        s_packed = m.stats()["s_packed"]
+    finally:
+        dist.barrier(group=gloo)
+        if rank != 0:  # consumers first: they read the producer's buffers
+            m.close()
+        dist.barrier(group=gloo)
+        if rank == 0:
+            m.close()
+        del tensors
+        torch.cuda.empty_cache()
+    return {"lat": lat, "host": host, "inst": inst, "verify": ver, "s_packed": s_packed}
+
+
+def gather_obj(obj, gloo):
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size(group=gloo)
+    dist.all_gather_object(out, obj, group=gloo)
+    return out
+
+
+def summarize_fanout(per_rank, S):
+    """Rank 0's view of one fan-out: value = the max over ranks of each rank's
+    device-timed update window (the producer's CUDA events bracket every
+    consumer's swap; a consumer's own window is its install kernel)."""
+    if any("unsupported" in r for r in per_rank):
+        return {"unsupported": next(r["unsupported"] for r in per_rank if "unsupported" in r)}
+    p = per_rank[0]
+    lat_ms = statistics.mean(p["lat"])
+    inst_us = [statistics.median(r["inst"]) if r["inst"] else 0.0 for r in per_rank[1:]]
+    win = max([lat_ms] + [u / 1e3 for u in inst_us])
+    ver = [r["verify"] for r in per_rank]
+    return {
+        "latency_ms": round(win, 6), "latency_p50_ms": round(statistics.median(p["lat"]), 6),
+        "latency_min_ms": round(min(p["lat"]), 6), "host_latency_ms": round(statistics.mean(p["host"]), 6),
+        "update_gbps_per_consumer": round(S / (win * 1e-3) / 1e9, 3),
+        "nvlink_frac": round(S / (win * 1e-3) / 1e9 / NVLINK_GBS, 4),
+        "install_kernel_us_per_consumer": [round(u, 3) for u in inst_us],
+        "install_kernel_nvlink_frac": round(S / (max(inst_us) * 1e-6) / 1e9 / NVLINK_GBS, 4) if max(inst_us) else None,
+        "parity": {"producer_seals_ok": ver[0]["seals_ok"],
+                   "consumers": [{"rank": i + 1, "seals_ok": v["seals_ok"], "bytes_ok": v["bytes_ok"],
+                                  "chunks": v["chunks"], "version_ok": v["version_ok"]} for i, v in enumerate(ver[1:])]},
+        "parity_ok": bool(ver[0]["seals_ok"] is not False and all(
+            v["seals_ok"] and v["bytes_ok"] and v["version_ok"] for v in ver[1:])),
+    }
+
+
+def xproc_concurrent(V, G, synth, name, rank, world, dev, gloo, fanout, seconds=2.0, period_ms=2.0):
+    """BASELINE.json configs[2] across processes: each consumer serves while
+    ASYNC updates land.  A reader thread per consumer loops acquire -> compare
+    every weight byte with VGEN(view.version) on its GPU -> stream-ordered
+    release; the producer publishes every `period_ms`.  Counts views, torn
+    views (must be 0) and version regressions; views/s idle vs during updates."""
+    import threading
+    import torch
+    import torch.distributed as dist
+    specs = synth.model_specs(name)
+    seed = synth.SEEDS[name]
+    tensors = G.alloc_model(specs)
+    bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
+    try:
+        m = V.Model(f"bench-xc-{name}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors, fanout=fanout,
+                    mode=V.ASYNC, device=dev, bootstrap=bs)
+    except V.ViperError as e:
+        return {"unsupported": f"{e.name}: {e.detail}"[:300]}
+    res = {"views_idle": 0.0, "views_busy": 0.0, "torn": 0, "regress": 0, "publishes": 0, "installs": 0}
+    try:
+        if rank == 0:
+            G.fill_model(tensors, specs, seed, 1)
+            m.publish(1)
+            torch.cuda.synchronize()
+        else:
+            m.wait_installed(1, timeout_us=30_000_000)
+        stop = threading.Event()
+        cnt = {"views": 0, "torn": 0, "regress": 0}
+
+        def reader():
+            torch.cuda.set_device(dev)
+            s = torch.cuda.Stream()
+            exp = G.alloc_model(specs, device=f"cuda:{dev}")
+            last = 0
+            with torch.cuda.stream(s):
+                while not stop.is_set():
+                    view = m.acquire_latest(timeout_us=100_000)
+                    G.fill_model(exp, specs, seed, view.version, stream=s)
+                    bad = torch.zeros((), dtype=torch.int64, device=f"cuda:{dev}")
+                    for g, e in zip(view.tensors(tensors), exp):
+                        bad += (g.view(torch.uint8) != e.view(torch.uint8)).sum()
+                    m.release(view, stream=s)
+                    cnt["torn"] += int(int(bad.item()) > 0)
+                    cnt["regress"] += int(view.version < last)
+                    last = view.version
+                    cnt["views"] += 1
+
+        for phase in ("idle", "busy"):
+            dist.barrier(group=gloo)
+            cnt["views"] = 0
+            th = threading.Thread(target=reader) if rank else None
+            if th:
+                th.start()
+            t0 = time.perf_counter()
+            if rank == 0:
+                v = m.stats()["version"]
+                ps = torch.cuda.Stream()
+                while time.perf_counter() - t0 < seconds:
+                    if phase == "busy":
+                        v += 1
+                        with torch.cuda.stream(ps):
+                            G.fill_model(tensors, specs, seed, v, stream=ps)
+                            m.publish(v, stream=ps)
+                        res["publishes"] += 1
+                    time.sleep(period_ms / 1e3)
+                ps.synchronize()
+                last_v = torch.tensor([float(v)])
+            else:
+                time.sleep(seconds)
+                last_v = torch.tensor([0.0])
+            dist.all_reduce(last_v, op=dist.ReduceOp.MAX, group=gloo)
+            if rank:
+                m.wait_installed(int(last_v.item()), timeout_us=60_000_000)
+                stop.set()
+                th.join()
+                stop.clear()
+                res[f"views_{phase}"] = cnt["views"] / (time.perf_counter() - t0)
+        res["torn"], res["regress"] = cnt["torn"], cnt["regress"]
+        if rank:
+            res["installs"] = m.stats()["installs"]
+    finally:
+        dist.barrier(group=gloo)
+        if rank != 0:
+            m.close()
+        dist.barrier(group=gloo)
+        if rank == 0:
+            m.close()
+        del tensors
+        torch.cuda.empty_cache()
+    return res
+
+
+def xproc_arm(args):
+    """N > 1: one process per GPU (self-launched by main() when WORLD_SIZE is
+    unset).  Rank 0 is the producer, ranks 1..N-1 the consumers.  The workload
+    follows BASELINE.json: N = 2 -> configs[1] ResNet-50 1 -> 1, N = 4 ->
+    configs[2] ViT-B/16 1 -> 3 with concurrent acquire, N = 8 -> configs[3]
+    GPT-2 XL 1 -> 7 (other N: ResNet-50).  Every fan-out the engine has is
+    timed on the same bytes (SYNC updates): the headline is NVLS where the box
+    exposes multicast, else scatter-allgather (N > 2) / direct pull (N = 2);
+    the others, push, chain, direct star and the engine's copy-engine baseline
+    sit beside it, with an NCCL broadcast and a torch copy-engine pull of the
+    same bytes as baselines.  Each fan-out's last version is verified on every
+    consumer against the oracle's golden chunk seals and byte for byte
+    (verify_replicas).  Roofline: f_NVL = (S / L_update) / 900 GB/s (SURVEY
+    s8(d)), the install kernel's own S / t_install beside it."""
+    import torch
+    import torch.distributed as dist
+    rank, world, local = dist_env()
+    if not torch.cuda.is_available() or torch.cuda.device_count() == 0:
+        # no GPU (CPU plumbing check of the launcher): rendezvous, max over
+        # ranks, one line from rank 0 -- and no number
+        dist.init_process_group("gloo")
+        t = torch.tensor([float(rank)])
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "value": None, "unit": "ms", "n_gpus": world, "steps": args.steps,
+                              "warmup": args.warmup, "higher_is_better": False, "scaling": "weak",
+                              "ranks_seen": int(t.item()) + 1,
+                              "unavailable": "no CUDA device visible: launcher / rendezvous / max-over-ranks "
+                                             "plumbing only, nothing measured"}), flush=True)
+        dist.barrier()
+        dist.destroy_process_group()
+        return
+    import synth
+    from synth import gpu as G
+    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+    ndev = torch.cuda.device_count()
+    over = ndev < world
+    if over and not args.oversubscribe:
+        raise SystemExit(f"bench.py: {world} ranks but {ndev} visible GPU(s); pass --oversubscribe to run the "
+                         f"code path with ranks sharing GPUs (no NVLink is measured then)")
+    dev = local % ndev
+    torch.cuda.set_device(dev)
+    if over:
+        dist.init_process_group("gloo")
+    else:
+        dist.init_process_group("cpu:gloo,cuda:nccl", device_id=torch.device("cuda", dev))
+    gloo = dist.new_group(backend="gloo")
+    name = args.config if args.config_explicit else N_CONFIG.get(world, "resnet50")
     S = synth.model_bytes(name)
+    flush = torch.empty(FLUSH_BYTES, dtype=torch.uint8, device="cuda")
+    # the fan-outs to time: headline first
+    if args.fanout != "auto":
+        order = [args.fanout]
+    elif world == 2:
+        order = ["direct", "push", "ce", "nvls"]
+    else:
+        order = ["nvls", "sa", "chain", "push", "direct", "ce"]
+    if over and args.fanout == "auto":  # ranks time-slice one GPU: peer waits only serialise (DESIGN.md s8)
+        order = ["direct", "push", "ce"]
+    results = {}
+    with ClockSampler(dev) as clk:
+        for f in order:
+            if f == "push" and world - 1 > 8:
+                continue
+            r = xproc_updates(V, G, synth, name, rank, world, dev, gloo, FANOUTS[f], flush, args.steps, args.warmup)
+            results[f] = summarize_fanout(gather_obj(r, gloo), S) if rank == 0 else None
+            dist.barrier(group=gloo)
+    head = next((f for f in order if rank != 0 or "unsupported" not in results[f]), order[0])
+    head = gather_obj(head, gloo)[0]
+    # baselines on the same bytes: NCCL broadcast (device time, max over ranks) and a torch copy-engine pull
     buf = torch.empty(S, dtype=torch.uint8, device="cuda")
-    nccl_ms = [float("nan")] if over else []
+    nccl_ms = []
     for i in range(0 if over else args.warmup + args.steps):
         torch.cuda.synchronize()
         dist.barrier()
@@ -700,47 +1065,65 @@ def xproc_arm(args):
             nccl_ms.append(e0.elapsed_time(e1))
     ce_ms = ce_baseline(rank, gloo, buf, args.steps, args.warmup)
     del buf
-    e2e = xproc_e2e(V, G, synth, name, rank, world, dev, gloo, fanout, flush, args.steps, args.warmup)
-    t = torch.tensor([statistics.mean(lat[args.warmup:]) if rank == 0 else 0.0,
-                      statistics.median(inst[args.warmup:]) if rank else 0.0,
-                      statistics.mean(nccl_ms), float(1 - ok), e2e["ms"], float(1 - e2e["ok"]), ce_ms],
+    torch.cuda.empty_cache()
+    conc = xproc_concurrent(V, G, synth, name, rank, world, dev, gloo, FANOUTS[head])
+    conc_all = gather_obj(conc, gloo)
+    e2e = xproc_e2e(V, G, synth, name, rank, world, dev, gloo, FANOUTS[head], flush, args.steps, args.warmup)
+    t = torch.tensor([statistics.mean(nccl_ms) if nccl_ms else 0.0, ce_ms, e2e["ms"], float(1 - e2e["ok"])],
                      dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
-    if rank != 0:
-        m.close()
-    dist.barrier(group=gloo)
     if rank == 0:
-        m.close()
         peak, peak_kind = load_peaks()
-        lat_ms, inst_us, nccl = float(t[0]), float(t[1]), float(t[2])
-        nvl = 770.0  # measured peer copy GB/s per direction (B200_PROFILING.md)
+        h = results[head]
+        ok = "unsupported" not in h
+        lat_ms = h["latency_ms"] if ok else None
+        inst = max(h["install_kernel_us_per_consumer"]) if ok else None
+        cons = [c for c in conc_all[1:] if "unsupported" not in c]
         out = {
-            "metric": METRIC, "value": round(lat_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": round(lat_ms, 6), "higher_is_better": False, "scaling": "weak",
+            "metric": METRIC, "value": lat_ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": lat_ms, "higher_is_better": False, "scaling": "weak",
             "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
             "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
-            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumers "
+            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumer(s) "
                                    f"{'sharing one GPU (code path only, no NVLink)' if over else 'over NVLink'} "
-                                   f"({fanout_name}), SYNC",
-                       "model_bytes": S, "devices_visible": ndev,
-                       "oversubscribed": ndev < world, "l2": "flushed before every update"},
-            "update_gbps_per_consumer": round(S / (lat_ms * 1e-3) / 1e9, 3),
-            "install_kernel_us_max_over_consumers": round(inst_us, 3),
-            "roofline": None if over else {
-                "bound": "nvlink", "kernel": "install_verify (peer pull)",
-                "achieved": round(S / (inst_us * 1e-6) / 1e9, 2), "peak": nvl, "unit": "GB/s",
-                "frac": round(S / (inst_us * 1e-6) / 1e9 / nvl, 4), "traffic": None,
-                "peak_kind": "measured peer copy (B200_PROFILING.md)"},
-            "nccl_broadcast_ms": None if over else round(nccl, 6),
-            "ce_pull_ms": round(float(t[6]), 6),
+                                   f"({FANOUT_NAMES[FANOUTS[head]]}), SYNC",
+                       "baseline_config": f"BASELINE.json configs[{CONFIG_INDEX[name]}]", "fanout": head,
+                       "model_bytes": S, "devices_visible": ndev, "oversubscribed": over,
+                       "l2": "flushed on every rank before every update (256 MiB write + 256 MiB read)",
+                       "parallelism": f"1 producer + {world - 1} consumers, one process per GPU"},
+            "update_gbps_per_consumer": h.get("update_gbps_per_consumer"),
+            "roofline": None if (over or not ok) else {
+                "bound": "nvlink", "kernel": "update: pack -> NVLink delivery -> install + verify + swap (pipelined)",
+                "achieved": round(S / (lat_ms * 1e-3) / 1e9, 2), "peak": NVLINK_GBS, "unit": "GB/s",
+                "frac": round(S / (lat_ms * 1e-3) / 1e9 / NVLINK_GBS, 4), "traffic": None,
+                "peak_kind": "NVLink 5 per direction per GPU (north_star; B200_PROFILING.md)",
+                "algorithmic_bytes": S, "formula": "f_NVL = (S / L_update) / 900 GB/s (SURVEY s8(d))",
+                "install_kernel": {"us": inst, "achieved": round(S / (inst * 1e-6) / 1e9, 2) if inst else None,
+                                   "frac": h["install_kernel_nvlink_frac"]}},
+            "fanouts": results,
+            "parity_ok": h.get("parity_ok", False),
+            "parity": h.get("parity"),
+            "nccl_broadcast_ms": None if over else round(float(t[0]), 6),
+            "ce_pull_ms": round(float(t[1]), 6),
             "ce_pull_how": "SURVEY B2 baseline: every consumer pulls the producer's S bytes at once with the copy "
                            "engine (torch copy_ from the CUDA-IPC-mapped producer buffer = cudaMemcpyPeerAsync), "
                            "CUDA events, max over consumers",
-            "parity_ok": bool(float(t[3]) == 0.0),
-            "gpu_launches": 3 * args.steps,
+            "concurrent_acquire": {
+                "how": f"ASYNC publish every 2 ms for 2 s ({FANOUT_NAMES[FANOUTS[head]]}); per consumer a reader "
+                       "thread acquires, compares every weight byte with VGEN(view.version) on its GPU, releases",
+                "torn_views": sum(c["torn"] for c in cons), "version_regressions": sum(c["regress"] for c in cons),
+                "views_per_s_idle": [round(c["views_idle"], 1) for c in cons],
+                "views_per_s_during_updates": [round(c["views_busy"], 1) for c in cons],
+                "publishes": conc_all[0].get("publishes"), "installs": [c["installs"] for c in cons],
+                **({"unsupported": conc_all[0]["unsupported"]} if "unsupported" in conc_all[0] else {})},
+            "gpu_launches": (2 + (world - 1)) * args.steps,
+            "gpu_launches_how": "per update: pack (+ push / NVLS stores) and seal_reduce on the producer, one "
+                                "install per consumer",
             "clocks": clk.summary(),
-            "e2e": {"value": round(float(t[4]), 6), "unit": "ms", "h2d_bytes_per_step": e2e["h2d"],
-                    "d2h_bytes_per_step": e2e["d2h"], "digest_ok": bool(float(t[5]) == 0.0),
+            "cpu_baseline": None,
+            "cpu_baseline_note": "the oracle is timed on rank 0 at N = 1 only (task rule); see the N = 1 line",
+            "e2e": {"value": round(float(t[2]), 6), "unit": "ms", "h2d_bytes_per_step": e2e["h2d"],
+                    "d2h_bytes_per_step": e2e["d2h"], "digest_ok": bool(float(t[3]) == 0.0),
                     "how": "rank 0: pinned host -> device copy of the step's weights, SYNC publish (returns "
                            "after every consumer swapped), D2H of the chunk-seal digest; host clock"},
         }
@@ -796,6 +1179,8 @@ def gpu_arm(args):
     dom, dom_us = "publish_fused (pack_seal + install_verify + swap)", fused
     achieved = alg / (dom_us * 1e-6) / 1e9
     calib = event_floor_us(G)
+    b2b_ms, b2b_ok = run_back_to_back(V, G, synth, name, args.steps, args.warmup)
+    gold = golden_check_local(V, G, synth, name)
     out = {
         "metric": METRIC, "value": round(mean_ms, 6), "unit": "ms", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": round(mean_ms, 6), "higher_is_better": False,
@@ -821,6 +1206,12 @@ def gpu_arm(args):
                      "fused_hbm_frac": round(alg / (fused_dirty * 1e-6) / 1e9 / peak, 4),
                      "how": "write-only 256 MiB flush: ~126 MB of dirty harness lines stay in L2 and are written "
                             "back during the timed kernel", "parity_ok": rd["ok"] and ktd["ok"]},
+        "latency_back_to_back_ms": round(b2b_ms, 6),
+        "back_to_back": {"hbm_frac": round(alg / (b2b_ms * 1e-3) / 1e9 / peak, 4), "parity_ok": b2b_ok,
+                         "how": "K SYNC publishes issued back to back, one CUDA-event window around all K (no flush, "
+                                "no optimizer write): each update pays the deferred L2 write-back of the previous "
+                                "one; 3S algorithmic bytes per update vs measured HBM"},
+        "parity_golden": gold,
         "kernels_us": {"publish_fused": round(fused, 3), "pack_seal": round(pack, 3),
                        "install_verify": round(inst, 3), "event_bracket_floor": round(calib, 3),
                        "how": "library CUDA events around each kernel, stream kept busy (no host gaps); "
@@ -833,7 +1224,7 @@ def gpu_arm(args):
                      "duration": "CUDA events around each launch on its stream (includes the event_bracket_floor)",
                      "ncu_launch_list": ncu_launches(name, "publish_fused_kernel", alg, peak),
                      "frac_of_nominal_7700": round(achieved / HBM_NOMINAL_GBS, 4)},
-        "parity_ok": r["ok"],
+        "parity_ok": bool(r["ok"] and gold["producer_seals_ok"] and gold["consumer_seals_ok"] and gold["bytes_ok"]),
         "gpu_launches": 2 * args.steps,  # publish_fused + seal_reduce per update
     }
     out["clocks"] = clk.summary()
@@ -912,12 +1303,23 @@ def gpu_arm(args):
 
 
 def reference_arm(args):
+    """The oracle on the host cores, on this arm's config: at N > 1 rank 0
+    alone runs it with the same 1 -> N-1 fan-out (N-1 oracle consumers, as
+    many as fit in 40% of the host's available memory; the sample says how
+    many), the other ranks exit without work."""
     rank, world, _ = dist_env()
     if rank != 0:
         return
     import synth
-    name = args.config
-    o = OracleUpdates(synth, name)
+    name = args.config if (args.config_explicit or world == 1) else N_CONFIG.get(world, "resnet50")
+    ncons = max(1, world - 1)
+    try:
+        avail = os.sysconf("SC_AVPHYS_PAGES") * os.sysconf("SC_PAGE_SIZE")
+        fit = int((0.4 * avail / synth.model_bytes(name) - 3) // 3)  # producer + 2 versions; 3 S per consumer
+        ncons = max(1, min(ncons, fit))
+    except (ValueError, OSError):
+        pass
+    o = OracleUpdates(synth, name, ncons=ncons)
     res = []
     try:
         for i in range(args.warmup + args.steps):
@@ -930,12 +1332,39 @@ def reference_arm(args):
     out = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "ms", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(v, 4), "higher_is_better": False,
            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
-           "data": "synthetic (VGEN)", "config": {"workload": f"{name}: 1 producer -> 1 consumer, the oracle on host cores "
-                                                     f"(BASELINE.json configs[{CONFIG_INDEX[name]}])"},
+           "data": "synthetic (VGEN)", "config": {"workload": f"{name}: 1 producer -> {ncons} consumer(s), the oracle on "
+                                                     f"host cores (BASELINE.json configs[{CONFIG_INDEX[name]}])"},
            "cpu_baseline": {"value": round(v, 4), "unit": "ms", "cores": 1, "kind": "oracle", "cpu": cpu_model(),
-                            "sample": "each step = up to 20 oracle updates, mean ms per update"},
+                            "sample": f"each step = up to 20 oracle updates to {ncons} consumer(s), mean ms per update"},
            "e2e": {"value": round(v, 4), "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
+
+
+def free_port() -> int:
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
+def launch_ranks(args) -> int:
+    """`--gpus N` (N > 1) without a launcher: start N ranks of this script with
+    torch.distributed.run on 127.0.0.1 (the same command the driver uses), one
+    per GPU.  Fails loudly when fewer than N GPUs are visible, unless
+    --oversubscribe (ranks then share GPUs: a code-path run, no NVLink)."""
+    ndev = 0
+    try:
+        import torch
+        ndev = torch.cuda.device_count() if torch.cuda.is_available() else 0
+    except Exception:
+        pass
+    if ndev < args.gpus and not args.oversubscribe:
+        print(f"bench.py: --gpus {args.gpus} but {ndev} GPU(s) visible (pass --oversubscribe to share GPUs)",
+              file=sys.stderr, flush=True)
+        return 2
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.run(cmd).returncode
 
 
 def main():
@@ -945,8 +1374,11 @@ def main():
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="viper", choices=["viper", "reference"])
     ap.add_argument("--config", default=None, choices=["ptychonn", "resnet50", "vit_b16", "gpt2_xl", "llama3_8b"])
-    ap.add_argument("--fanout", default="auto", choices=["auto", "direct", "chain", "sa"],
-                    help="N > 2 fan-out (auto: direct for one consumer, scatter-allgather for more)")
+    ap.add_argument("--fanout", default="auto", choices=["auto"] + sorted(FANOUTS),
+                    help="N > 1: time only this fan-out (auto: every fan-out, headline NVLS where available, else "
+                         "scatter-allgather for N > 2 and direct pull for N = 2)")
+    ap.add_argument("--oversubscribe", action="store_true",
+                    help="N > 1 with fewer visible GPUs than ranks: ranks share GPUs (code path only, no NVLink)")
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     args = ap.parse_args()
@@ -954,6 +1386,13 @@ def main():
     args.config_explicit = args.config is not None
     if args.config is None:
         args.config = "resnet50"  # BASELINE.json configs[1] (1-GPU loopback)
+    if args.gpus < 1:
+        raise SystemExit("bench.py: --gpus must be >= 1")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(launch_ranks(args))  # one process per GPU, then each rank re-enters main()
+    _, world, _ = dist_env()
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
     if args.impl == "reference":
         reference_arm(args)
     else:

@@ -111,8 +111,34 @@ enum { VIPER_FANOUT_DIRECT = 0,        /* every consumer pulls every chunk from 
                                           soon as that item is sealed there, and stages it
                                           for consumer i+1.  Producer egress S; bound
                                           S/link + (N-1) items (SURVEY s8(e) option 3) */
-       VIPER_FANOUT_SCATTER_ALLGATHER = 2 /* consumer i pulls chunks c = i (mod N) from the
-                                             producer, the rest from its peers */ };
+       VIPER_FANOUT_SCATTER_ALLGATHER = 2, /* consumer i pulls chunks c = i (mod N) from the
+                                             producer, the rest from its peers */
+       VIPER_FANOUT_NVLS = 3,          /* NVSwitch multicast (SURVEY s8(e) option 1): every
+                                          rank binds a staging buffer to one multicast
+                                          object; the producer's pack stores each item
+                                          once into the multicast address
+                                          (multimem.st), the switch replicates it to every
+                                          consumer, and each consumer installs from its own
+                                          HBM.  Producer egress S.  Needs a GPU tier, one
+                                          GPU per rank and cuMulticastCreate support
+                                          (fabric manager); otherwise registration returns
+                                          VIPER_E_UNSUPPORTED on every rank */
+       VIPER_FANOUT_PUSH = 4,          /* push (SURVEY K3 deliver_push): the producer's
+                                          pack stores every item into each consumer's
+                                          peer-mapped staging as well as its snapshot
+                                          (producer egress N x S, at most 8 consumers);
+                                          consumers install from local HBM, item by item
+                                          as the producer releases the item seals */
+       VIPER_FANOUT_NCCL = 100,        /* baseline: reserved; bench.py times
+                                          torch.distributed.broadcast over NCCL instead.
+                                          Registration returns VIPER_E_UNSUPPORTED */
+       VIPER_FANOUT_CE = 101           /* baseline: each consumer's update
+                                          thread copies the sealed snapshot with the copy
+                                          engine (cudaMemcpyAsync peer -> local staging)
+                                          once the pack completed, then installs locally */
+};
+/* NVLS, PUSH and CE are cross-process fan-outs (viper_bootstrap != NULL, GPU
+ * tier, one producer); in process they return VIPER_E_UNSUPPORTED. */
 /* Save mode (Fig. 3; s5.3 P:2143-2153). */
 enum { VIPER_SYNC = 0,   /* publish returns after every consumer installed v (or failed) */
        VIPER_ASYNC = 1 };/* publish returns once the snapshot is enqueued on cuda_stream;
@@ -277,6 +303,21 @@ viper_status viper_get_stats(viper_model *m, viper_stats *out);
  * DRAM-tier staging buffer (NULL on the GPU tier) and NULL seals. */
 viper_status viper_layout(viper_model *m, uint64_t *s_packed, uint64_t *offsets, int32_t n);
 viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_seals, uint64_t *nchunks);
+
+/*
+ * viper_view_seals -- consumer: the chunk seals of a pinned view, computed on
+ * the device from the installed slot tensors as they sit (no copy).  Output:
+ * nchunks x {uint64 version = view->version, uint64 cks} in dev_seals_out, a
+ * caller-owned device buffer of >= 16 * nchunks bytes on the model's device,
+ * written in stream order on cuda_stream (the caller synchronises before
+ * reading it).  cks is the CKS of DESIGN.md R16 over the packed layout (LAY,
+ * zero padding), i.e. the value the producer sealed chunk c with, so equality
+ * with the producer's (or the oracle's) chunk seals proves the replica
+ * byte-exact up to the checksum's guarantees ("the updated model ... replaces
+ * the previous model", s4.2 P:1208-1227).  The view must stay pinned until the
+ * stream passes the call.  VIPER_E_STATE: producer / unknown view.
+ */
+viper_status viper_view_seals(viper_model *m, const viper_view *view, void *dev_seals_out, void *cuda_stream);
 
 /* Test hook (T4 fault injection): the consumer's next install flips one
  * staged bit before verification -> VIPER_E_CHECKSUM, version not installed. */

@@ -17,7 +17,7 @@ CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libviper.so")
 VGEN_SRC = os.path.join(ROOT, "synth", "vgen.cu")
 VGEN_LIB = os.path.join(ROOT, "synth", "libvgen.so")
-SOURCES = ["kernels.cu", "runtime.cpp", "schedule.cpp", "xproc.cpp", "flush.cpp", "selftest.cpp"]
+SOURCES = ["kernels.cu", "runtime.cpp", "schedule.cpp", "xproc.cpp", "flush.cpp", "selftest.cpp", "nvls.cpp"]
 HEADERS = ["vp_internal.h", "runtime.h", "protocol.h", "selector.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

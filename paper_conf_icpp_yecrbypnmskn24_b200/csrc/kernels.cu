@@ -167,7 +167,7 @@ __device__ __forceinline__ uint64_t copy_words_bytewise(const uint8_t *__restric
 
 // Copy one work item (src -> dst, n bytes, packed offset p0); returns the
 // lane's partial checksum of the packed-space words it moved.
-template <bool kCoherent>
+template <bool kCoherent, int U = kUnroll>
 __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst, uint32_t n,
                                               uint64_t p0, uint32_t lane, bool inject) {
     uint64_t acc = 0;
@@ -175,16 +175,16 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
     if (!aligned) return copy_words_bytewise<kCoherent>(src, dst, 0, n, p0, lane, inject);
     const uint32_t nvec = n >> 4;
     const uint32_t g0 = (uint32_t)(p0 >> 2);
-    for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
-        uint4 r[kUnroll];
+    for (uint32_t base = 0; base < nvec; base += 32 * U) {
+        uint4 r[U];
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
+        for (int u = 0; u < U; u++) {
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) r[u] = kCoherent ? ld_cg(src + (size_t)i * 16) : ld_stream(src + (size_t)i * 16);
         }
         if (inject && base == 0 && lane == 0) r[0].x ^= 0x10u;
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
+        for (int u = 0; u < U; u++) {
             const uint32_t i = base + u * 32 + lane;
             if (i < nvec) {
                 st_v4(dst + (size_t)i * 16, r[u]);
@@ -299,6 +299,153 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
     }
 }
 
+// ---------------------------------------------------------------------------
+// Push delivery (VIPER_FANOUT_PUSH): the pack stores every item into
+// its local snapshot AND straight into each consumer's peer-mapped staging
+// (NVLink stores: fire-and-forget, so the warp streams at the link rate), then
+// releases the item's seal at system scope in every staging.  Consumers install
+// from their own HBM, item by item behind these seals.
+__device__ __forceinline__ uint64_t copy_item_push(const uint8_t *__restrict__ src, uint8_t *__restrict__ snap,
+                                                   const PushArgs &a, uint64_t off, uint32_t n, uint32_t lane) {
+    bool aligned = (((uintptr_t)src | (uintptr_t)snap) & 15u) == 0;
+    if (!aligned) {  // rare (unaligned source tensor): word path, then copy the snapshot piece out
+        const uint64_t acc = copy_words_bytewise<false>(src, snap, 0, n, off, lane, false);
+        __syncwarp();
+        for (uint32_t k = 0; k < a.ndst; k++) copy_words_bytewise<true>(snap, a.dst[k] + off, 0, n, off, lane, false);
+        return acc;
+    }
+    uint64_t acc = 0;
+    const uint32_t nvec = n >> 4;
+    const uint32_t g0 = (uint32_t)(off >> 2);
+    for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
+        uint4 r[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            const uint32_t i = base + u * 32 + lane;
+            if (i < nvec) r[u] = ld_stream(src + (size_t)i * 16);
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            const uint32_t i = base + u * 32 + lane;
+            if (i < nvec) {
+                st_v4(snap + (size_t)i * 16, r[u]);
+                acc += cks_vec(r[u], g0 + 4u * i);
+            }
+        }
+        for (uint32_t k = 0; k < a.ndst; k++) {
+            uint8_t *d = a.dst[k] + off;
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) st_v4(d + (size_t)i * 16, r[u]);
+            }
+        }
+    }
+    if (n & 15u) {  // < 16-B tensor tail (packed offsets are 16-B aligned, the tail is not)
+        acc += copy_words_bytewise<false>(src, snap, nvec * 16, n, off, lane, false);
+        __syncwarp();
+        for (uint32_t k = 0; k < a.ndst; k++) copy_words_bytewise<true>(snap, a.dst[k] + off, nvec * 16, n, off, lane, false);
+    }
+    return acc;
+}
+
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_push_kernel(const PushArgs a) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.p.nitems; w += nwarps) {
+        const Item it = a.p.items[w];
+        const uint64_t part = warp_sum(copy_item_push((const uint8_t *)it.ptr, a.p.packed + it.packed_off, a,
+                                                      it.packed_off, it.nbytes, lane));
+        __syncwarp();  // every lane's stores are ordered before lane 0's releases
+        if (lane == 0) {
+            const uint64_t mixed = part + a.p.version * kVerMix;
+            a.p.iseal[it.gidx].mixed = mixed;
+            st_release(&a.p.iseal[it.gidx].version, a.p.version);
+            for (uint32_t k = 0; k < a.ndst; k++) {  // the consumers' copies of the seal, after the data
+                a.dst_iseal[k][it.gidx].mixed = mixed;
+                st_release_sys(&a.dst_iseal[k][it.gidx].version, a.p.version);
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// NVLS multicast delivery (VIPER_FANOUT_NVLS): the snapshot lives in
+// memory bound to one multicast object on every rank; the pack stores each
+// 16-B vector once to the multicast address (multimem.st) and NVSwitch writes
+// it into the producer's snapshot and every consumer's staging.  The item seal
+// follows with a system-scope release through the same multicast address.
+__device__ __forceinline__ void mc_st_v4(void *p, const uint4 &v) {
+    asm volatile("multimem.st.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mc_st_u32(void *p, uint32_t v) {
+    asm volatile("multimem.st.global.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void mc_st_u64(void *p, uint64_t v) {
+    asm volatile("multimem.st.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void mc_st_release_sys_u64(void *p, uint64_t v) {
+    asm volatile("multimem.st.release.sys.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_nvls_kernel(const NvlsArgs a) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        const uint8_t *src = (const uint8_t *)it.ptr;
+        uint8_t *dst = a.mc_packed + it.packed_off;
+        const uint32_t n = it.nbytes;
+        uint64_t acc = 0;
+        uint32_t done = 0;
+        if (((uintptr_t)src & 15u) == 0) {
+            const uint32_t nvec = n >> 4;
+            const uint32_t g0 = (uint32_t)(it.packed_off >> 2);
+            for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
+                uint4 r[kUnroll];
+#pragma unroll
+                for (int u = 0; u < kUnroll; u++) {
+                    const uint32_t i = base + u * 32 + lane;
+                    if (i < nvec) r[u] = ld_stream(src + (size_t)i * 16);
+                }
+#pragma unroll
+                for (int u = 0; u < kUnroll; u++) {
+                    const uint32_t i = base + u * 32 + lane;
+                    if (i < nvec) {
+                        mc_st_v4(dst + (size_t)i * 16, r[u]);
+                        acc += cks_vec(r[u], g0 + 4u * i);
+                    }
+                }
+            }
+            done = nvec * 16;
+        }
+        // word path (unaligned source or < 16-B tail): whole little-endian words;
+        // the bytes past n in the last word are padding, which is zero by LAY
+        for (uint32_t wd = done / 4 + lane; wd * 4 < n; wd += 32) {
+            uint32_t word = 0;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const uint32_t b = wd * 4 + k;
+                if (b < n) word |= (uint32_t)src[b] << (8 * k);
+            }
+            mc_st_u32(dst + wd * 4, word);
+            const uint32_t g = (uint32_t)((it.packed_off + wd * 4) >> 2);
+            acc += (uint64_t)(word * ((2u * g + 1u) * kCksK));
+        }
+        const uint64_t part = warp_sum(acc);
+        __syncwarp();
+        if (lane == 0) {
+            mc_st_u64(&a.mc_iseal[it.gidx].mixed, part + a.version * kVerMix);
+            asm volatile("fence.acq_rel.sys;" ::: "memory");
+            mc_st_release_sys_u64(&a.mc_iseal[it.gidx].version, a.version);
+        }
+    }
+}
+
 // chunk seals {version, sum of item checksums} -- one warp per chunk, off the
 // critical path (side stream); they are what DESIGN.md R16 / the oracle define.
 __global__ void seal_reduce_kernel(const SealReduceArgs a) {
@@ -313,6 +460,62 @@ __global__ void seal_reduce_kernel(const SealReduceArgs a) {
     if (lane == 0) {
         a.seals[c].cks = s;
         a.seals[c].version = a.version;
+    }
+}
+
+// Checksum of one item read in place (no copy): the CKS terms of the packed
+// words it covers (any alignment; words zero-extended past n).
+__device__ __forceinline__ uint64_t cks_item_inplace(const uint8_t *__restrict__ src, uint32_t n, uint64_t p0,
+                                                     uint32_t lane) {
+    uint64_t acc = 0;
+    uint32_t done = 0;
+    if (((uintptr_t)src & 15u) == 0) {
+        const uint32_t nvec = n >> 4;
+        const uint32_t g0 = (uint32_t)(p0 >> 2);
+        for (uint32_t base = 0; base < nvec; base += 32 * kUnroll) {
+            uint4 r[kUnroll];
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) r[u] = ld_cg(src + (size_t)i * 16);
+            }
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t i = base + u * 32 + lane;
+                if (i < nvec) acc += cks_vec(r[u], g0 + 4u * i);
+            }
+        }
+        done = nvec * 16;
+    }
+    for (uint32_t w = done / 4 + lane; w * 4 < n; w += 32) {
+        uint32_t word = 0;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint32_t b = w * 4 + k;
+            if (b < n) word |= (uint32_t)__ldcg(src + b) << (8 * k);
+        }
+        const uint32_t g = (uint32_t)((p0 + w * 4) >> 2);
+        acc += (uint64_t)(word * ((2u * g + 1u) * kCksK));
+    }
+    return acc;
+}
+
+// Chunk seals {version, cks} (R16) of a consumer slot as it is laid
+// out in place (viper_view_seals): the same CKS as the producer's snapshot
+// seals, computed from the installed tensors, so a consumer can prove its
+// replica byte-exact against the oracle's seals without a host copy.  `seals`
+// must be zeroed; item checksums are summed with 64-bit atomics (the sum is
+// commutative, so the result is exact in any order).
+__global__ void __launch_bounds__(kWarpsPerBlock * 32) view_seal_kernel(const ViewSealArgs a) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
+        const Item it = a.items[w];
+        const uint64_t part = warp_sum(cks_item_inplace((const uint8_t *)it.ptr, it.nbytes, it.packed_off, lane));
+        if (lane == 0) {
+            atomicAdd((unsigned long long *)&a.seals[it.chunk].cks, (unsigned long long)part);
+            a.seals[it.chunk].version = a.version;
+        }
     }
 }
 
@@ -337,6 +540,13 @@ __device__ __forceinline__ bool grid_arrive(unsigned long long *flags, uint32_t 
     return true;
 }
 
+// A seal wait should stop: the host aborted the install (abort_h) or another
+// warp of this grid already timed out (its error bit is in the completion word).
+__device__ __forceinline__ bool wait_aborted(const InstallArgs &a) {
+    if (a.abort_h && *a.abort_h) return true;
+    return (*(volatile unsigned long long *)a.flags >> 32) & kErrTimeout;
+}
+
 // End of an install grid: the last block to finish publishes the result and,
 // when every item matched, swaps the version word from the device.
 __device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
@@ -346,8 +556,13 @@ __device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
     if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
         const int32_t st = (e & kErrTimeout) ? -6 : ((e & kErrChecksum) ? -5 : 0);
         // Every block's slot stores are GPU-visible (released by its arrival,
-        // acquired by this one); later readers are kernels launched after the
-        // host saw the flip, so plain system-visible stores suffice here.
+        // acquired by this one), which is all a reader on this GPU needs: it
+        // launches its kernels after the host saw the flip.  When the slot
+        // lives on ANOTHER GPU (an in-process SYNC install launched on the
+        // producer's stream), a system-scope fence -- cumulative over what
+        // this thread observed -- orders every block's peer stores before the
+        // swap becomes visible.
+        if (a.sys_swap) asm volatile("fence.acq_rel.sys;" ::: "memory");
         if (a.status_h) *a.status_h = st;
         if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
         if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
@@ -431,7 +646,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                 __nanosleep(backoff);
                 waited += backoff;
                 if (backoff < 1024) backoff <<= 1;
-                if (waited > kItemWaitNs) {  // never hang on a vanished producer
+                // never hang on a vanished producer: give up after kItemWaitNs,
+                // at once when the host aborts, or when another warp timed out
+                if (waited > kItemWaitNs || wait_aborted(a)) {
                     report_err(a.flags, kErrTimeout);
                     break;
                 }
@@ -477,6 +694,74 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
         }
         w = q.next(w, lane);
         if (w < a.nitems) q.claim(lane);
+    }
+    install_finish(a, bad);
+}
+
+// install_direct: the install of a COMPLETE snapshot (nothing left to wait
+// for: not PDL-chained, not early-notified) from one source -- the local or
+// NVLink-peer-mapped snapshot, or this GPU's staging (push / NVLS / CE / DRAM
+// tier).  The pack's structure: static item striding, and the next item's
+// descriptor AND its seal {cks, version} fetched one item ahead, so a warp's
+// only dependent round trip per item is its data.  The source is immutable
+// for the grid's lifetime (the consumer pins it), so the data is read with
+// non-coherent streaming loads.  A seal that does not show `version` yet (it
+// cannot, for a complete snapshot, but the kernel never trusts that) falls
+// back to the acquire spin of install_verify_kernel.
+__device__ __forceinline__ ISeal ld_seal(const ISeal *p) {
+    ISeal s;
+    asm volatile("ld.global.cg.v2.u64 {%0,%1}, [%2];" : "=l"(s.mixed), "=l"(s.version) : "l"(p));
+    return s;
+}
+
+#ifndef VP_ID_UNROLL
+#define VP_ID_UNROLL 8
+#endif
+#ifndef VP_ID_BLOCKS
+#define VP_ID_BLOCKS 2
+#endif
+constexpr int kIdUnroll = VP_ID_UNROLL;  // install_direct's own geometry (sweep: profiles/r02)
+constexpr int kIdBlocks = VP_ID_BLOCKS;
+
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kIdBlocks) install_direct_kernel(const InstallArgs a) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    bool bad = false;
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    Item nxt{};
+    ISeal nseal{};
+    if (w < a.nitems) {
+        nxt = a.items[w];
+        if (lane == 0) nseal = ld_seal(a.iseal + w);
+    }
+    for (; w < a.nitems; w += nwarps) {
+        const Item it = nxt;
+        uint64_t expect = 0;
+        if (lane == 0) {
+            if (nseal.version != a.version) {  // not expected for a complete snapshot: wait like install_verify
+                uint32_t backoff = 32;
+                uint64_t waited = 0;
+                while (ld_acquire_sys(&a.iseal[w].version) != a.version) {
+                    __nanosleep(backoff);
+                    waited += backoff;
+                    if (backoff < 1024) backoff <<= 1;
+                    if (waited > kItemWaitNs || wait_aborted(a)) {
+                        report_err(a.flags, kErrTimeout);
+                        break;
+                    }
+                }
+                nseal.mixed = a.iseal[w].mixed;
+            }
+            expect = nseal.mixed;
+        }
+        const uint32_t wn = w + nwarps;  // prefetch: its loads overlap this item's stream
+        if (wn < a.nitems) {
+            nxt = a.items[wn];
+            if (lane == 0) nseal = ld_seal(a.iseal + wn);
+        }
+        const uint64_t part = warp_sum(copy_item<false, kIdUnroll>(a.packed + it.packed_off, (uint8_t *)it.ptr,
+                                                                   it.nbytes, it.packed_off, lane, w == a.fault_item));
+        if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
     }
     install_finish(a, bad);
 }
@@ -550,6 +835,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
     uint32_t e;
     if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
         *reinterpret_cast<unsigned int *>(a.flags + 1) = 0;  // work counter: every warp stopped claiming
+        if (a.sys_swap) asm volatile("fence.acq_rel.sys;" ::: "memory");  // peer slots: see install_finish
         for (uint32_t k = 0; k < a.ncons; k++) {
             const FusedCons &c = a.cons[k];
             const int32_t st = (e >> k) & 1u ? -5 : 0;
@@ -798,7 +1084,7 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
             uint64_t waited = 0;
             while (ld_acquire_sys(&is->version) != a.version) {
                 __nanosleep(256);
-                if ((waited += 256) > kItemWaitNs) {
+                if ((waited += 256) > kItemWaitNs || wait_aborted(a)) {
                     report_err(a.flags, kErrTimeout);
                     break;
                 }
@@ -1052,6 +1338,7 @@ __global__ void __launch_bounds__(kFtWarps * 32, 2) publish_fused_tma_kernel(con
     __syncthreads();
     uint32_t e;
     if (threadIdx.x == 0 && grid_arrive(a.flags, &e)) {
+        if (a.sys_swap) asm volatile("fence.acq_rel.sys;" ::: "memory");  // peer slots: see install_finish
         for (uint32_t k = 0; k < a.ncons; k++) {
             const FusedCons &c = a.cons[k];
             const int32_t st = (e >> k) & 1u ? -5 : 0;
@@ -1087,8 +1374,18 @@ static int sm_count(int device) {
     return n;
 }
 
+// The launch runs on the CURRENT device (a SYNC publish launches a consumer's
+// install on the producer's stream), so both facts are keyed on it, not on
+// the endpoint's device.
+static int launch_device() {
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+
 template <typename Kernel>
-static cudaError_t opt_in_smem(Kernel kernel, size_t smem, int device, std::atomic<uint64_t> &done) {
+static cudaError_t opt_in_smem(Kernel kernel, size_t smem, int /*endpoint device*/, std::atomic<uint64_t> &done) {
+    const int device = launch_device();
     const uint64_t bit = 1ull << (device >= 0 && device < kMaxDevices ? device : 0);
     if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
     const cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1110,13 +1407,13 @@ FusedLaunch fused_tma_launch(uint32_t nitems, int device) {
     l.func = (const void *)publish_fused_tma_kernel;
     l.smem = kFtWarps * kFtStages * kFtStage + kFtWarps * kFtStages * sizeof(uint64_t);
     l.err = opt_in_smem(publish_fused_tma_kernel, l.smem, device, opted);
-    l.grid = grid_for(nitems, kFtWarps, sm_count(device), 2);
+    l.grid = grid_for(nitems, kFtWarps, sm_count(launch_device()), 2);
     l.block = kFtWarps * 32;
     return l;
 }
 
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
-    const int sms = sm_count(device);
+    const int sms = sm_count(launch_device());
     Geometry g;
     g.items = nitems;
     g.block = kWarpsPerBlock * 32;
@@ -1135,7 +1432,7 @@ cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
     static std::atomic<uint64_t> opted{0};
     const cudaError_t e = opt_in_smem(pack_seal_tma_kernel, kTmaSmem, device, opted);
     if (e != cudaSuccess) return e;
-    pack_seal_tma_kernel<<<grid_for(a.nitems, kTmaWarps, sm_count(device), 2), kTmaWarps * 32, kTmaSmem, st>>>(a);
+    pack_seal_tma_kernel<<<grid_for(a.nitems, kTmaWarps, sm_count(launch_device()), 2), kTmaWarps * 32, kTmaSmem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1144,7 +1441,7 @@ const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
 Geometry fused_geometry(const Geometry &g, int device) {
     // same block shape, up to kFusedBlocks resident blocks per SM
     Geometry f = g;
-    f.grid = grid_for(g.items, kWarpsPerBlock, sm_count(device), kFusedBlocks);
+    f.grid = grid_for(g.items, kWarpsPerBlock, sm_count(launch_device()), kFusedBlocks);
     return f;
 }
 
@@ -1157,7 +1454,7 @@ cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device
     static std::atomic<uint64_t> opted{0};
     const cudaError_t e = opt_in_smem(install_verify_tma_kernel, kTmaSmem, device, opted);
     if (e != cudaSuccess) return e;
-    const int sms = sm_count(device);
+    const int sms = sm_count(launch_device());
     const int grid = grid_for(a.nitems, kTmaWarps, max_sms > 0 && max_sms < sms ? max_sms : sms, 2);
     install_verify_tma_kernel<<<grid, kTmaWarps * 32, kTmaSmem, st>>>(a);
     return cudaGetLastError();
@@ -1169,7 +1466,7 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
         static std::atomic<uint64_t> opted{0};
         l.func = (const void *)pack_seal_tma_kernel;
         l.err = opt_in_smem(pack_seal_tma_kernel, kTmaSmem, device, opted);
-        l.grid = grid_for(a.nitems, kTmaWarps, sm_count(device), 2);
+        l.grid = grid_for(a.nitems, kTmaWarps, sm_count(launch_device()), 2);
         l.block = kTmaWarps * 32;
         l.smem = kTmaSmem;
     } else {
@@ -1180,11 +1477,16 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
     return l;
 }
 
-LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms) {
+LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms, bool direct) {
     LaunchSpec l{};
-    if (tma) {
+    if (direct && !tma) {
+        const int sms = sm_count(launch_device());
+        l.func = (const void *)install_direct_kernel;
+        l.grid = grid_for(a.nitems, kWarpsPerBlock, max_sms > 0 && max_sms < sms ? max_sms : sms, kIdBlocks);
+        l.block = g.block;
+    } else if (tma) {
         static std::atomic<uint64_t> opted{0};
-        const int sms = sm_count(device);
+        const int sms = sm_count(launch_device());
         l.func = (const void *)install_verify_tma_kernel;
         l.err = opt_in_smem(install_verify_tma_kernel, kTmaSmem, device, opted);
         l.grid = grid_for(a.nitems, kTmaWarps, max_sms > 0 && max_sms < sms ? max_sms : sms, 2);
@@ -1195,6 +1497,22 @@ LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int
         l.grid = g.grid;
         l.block = g.block;
     }
+    return l;
+}
+
+LaunchSpec push_launch(const Geometry &g) {
+    LaunchSpec l{};
+    l.func = (const void *)pack_push_kernel;
+    l.grid = g.grid;
+    l.block = g.block;
+    return l;
+}
+
+LaunchSpec nvls_launch(const Geometry &g) {
+    LaunchSpec l{};
+    l.func = (const void *)pack_nvls_kernel;
+    l.grid = g.grid;
+    l.block = g.block;
     return l;
 }
 
@@ -1209,6 +1527,49 @@ LaunchSpec seal_reduce_launch(const SealReduceArgs &a) {
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st) {
     if (a.nchunks == 0) return cudaSuccess;
     seal_reduce_kernel<<<(a.nchunks + 7) / 8, 256, 0, st>>>(a);
+    return cudaGetLastError();
+}
+
+// Load every kernel of the library into the current device's context now,
+// at registration, instead of at its first launch (CUDA lazy loading).  A lazy
+// load must wait for work already queued on the device, so the first launch
+// of an install behind a stream that waits for a producer (DRAM-tier piece
+// flags, an early-notified pack) could block the host thread for as long as
+// that producer takes -- forever if it died.  Once per device.
+cudaError_t preload_kernels() {
+    static std::atomic<uint64_t> done{0};
+    const int dev = launch_device();
+    const uint64_t bit = 1ull << (dev >= 0 && dev < kMaxDevices ? dev : 0);
+    if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+    const void *fns[] = {(const void *)pack_seal_kernel,         (const void *)seal_reduce_kernel,
+                         (const void *)install_verify_kernel,    (const void *)install_direct_kernel,
+                         (const void *)publish_fused_kernel,     (const void *)pack_seal_tma_kernel,
+                         (const void *)install_verify_tma_kernel, (const void *)publish_fused_tma_kernel,
+                         (const void *)view_seal_kernel,         (const void *)pack_push_kernel,
+                         (const void *)pack_nvls_kernel};
+    for (const void *f : fns) {
+        cudaFuncAttributes fa;
+        const cudaError_t e = cudaFuncGetAttributes(&fa, f);
+        if (e != cudaSuccess) return e;
+    }
+    // and the dynamic shared-memory opt-in of the TMA kernels (idempotent)
+    const size_t ft = kFtWarps * kFtStages * kFtStage + kFtWarps * kFtStages * sizeof(uint64_t);
+    cudaError_t e = cudaFuncSetAttribute(pack_seal_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(install_verify_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(publish_fused_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ft);
+    if (e != cudaSuccess) return e;
+    done.fetch_or(bit, std::memory_order_acq_rel);
+    return cudaSuccess;
+}
+
+cudaError_t launch_view_seals(const ViewSealArgs &a, cudaStream_t st) {
+    if (a.nitems == 0) return cudaSuccess;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    view_seal_kernel<<<grid_for(a.nitems, kWarpsPerBlock, sm_count(dev), kBlocksPerSM), kWarpsPerBlock * 32, 0, st>>>(
+        a);
     return cudaGetLastError();
 }
 

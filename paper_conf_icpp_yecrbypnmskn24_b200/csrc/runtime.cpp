@@ -11,7 +11,9 @@
 
 #include <cuda.h>  // types of the driver entry points (no libcuda link)
 #include <nvtx3/nvToolsExt.h>  // header-only; ranges cost nothing unless a tool attaches
+#include <errno.h>
 #include <linux/futex.h>
+#include <signal.h>
 #include <sched.h>
 #include <sys/syscall.h>
 #include <time.h>
@@ -361,11 +363,13 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
     pi->waited_us = (now_ns() - t0) / 1e3;
     InstallArgs &a = pi->a;
     a = InstallArgs{};
-    const bool dram = c->cfg.tier == VIPER_TIER_DRAM;
+    // DRAM tier / copy-engine baseline: the install reads this GPU's staging,
+    // filled by the copies launch_prepared enqueues ahead of the kernel
+    const bool staged = c->cfg.tier == VIPER_TIER_DRAM || c->cfg.fanout == VIPER_FANOUT_CE;
     a.items = c->d_slot_items[target];
     a.nitems = (uint32_t)c->man.items.size();
-    a.packed = dram ? c->d_stage : src.snap[b];
-    a.iseal = dram ? c->d_stage_iseal : src.iseal[b];
+    a.packed = staged ? c->d_stage : src.snap[b];
+    a.iseal = staged ? c->d_stage_iseal : src.iseal[b];
     a.version = v;
     a.target = (uint32_t)target;
     a.fault_item = ~0u;
@@ -375,6 +379,7 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
     a.status_h = (volatile int32_t *)&c->rec_dev->status;
     a.pin_h = (volatile uint64_t *)&c->rec_dev->pin;
     a.state_h = (volatile uint64_t *)&c->rec_dev->state;
+    a.abort_h = (const volatile int32_t *)&c->rec_dev->abort;
     return VIPER_OK;
 }
 
@@ -389,8 +394,15 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
         // staging, piece by piece as the producer's D2H lands (GPU-side waits
         // on the pieces' flags: the D2H and this H2D overlap)
         const Manifest &mm = c->man;
+        static const bool dbg = getenv("VIPER_DEBUG") != nullptr;
+        if (dbg) {
+            cudaPointerAttributes pa{};
+            cudaPointerGetAttributes(&pa, src.h_stage[b]);
+            fprintf(stderr, "[viper] DRAM install: %zu pieces, staging type %d\n", mm.piece_lo.size(), (int)pa.type);
+        }
         for (size_t i = 0; i < mm.piece_lo.size(); i++) {
             viper_status s = stream_wait_geq(st, &c->ctrl_dev->dram_flag[b][i], pi.a.version);
+            if (dbg) fprintf(stderr, "[viper]  piece %zu: wait enqueued (%d)\n", i, s);
             if (s) return s;
             CUDA_TRY(cudaMemcpyAsync(c->d_stage + mm.piece_lo[i], src.h_stage[b] + mm.piece_lo[i],
                                      mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyHostToDevice, st));
@@ -399,6 +411,15 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
         // raises the last flag after their D2H); only the install reads them
         CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.h_iseal[b], sizeof(ISeal) * mm.items.size(),
                                  cudaMemcpyHostToDevice, st));
+        if (dbg) fprintf(stderr, "[viper]  copies enqueued\n");
+        pdl = false;
+    } else if (c->cfg.fanout == VIPER_FANOUT_CE) {
+        // copy-engine baseline: the sealed snapshot (notified only
+        // once the pack completed) -> this GPU's staging over the peer
+        // mapping, then the same local install + verify
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage, src.snap[b], c->man.s_packed, cudaMemcpyDefault, st));
+        CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.iseal[b], sizeof(ISeal) * c->man.items.size(),
+                                 cudaMemcpyDefault, st));
         pdl = false;
     } else if (wait_ready && src.ev_ready[b]) {
         CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
@@ -411,11 +432,21 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     const bool direct = pi.a.sa_n == 0 && pi.a.mp_n <= 1;
     pi.a.l2_once = fits_l2(c->device, c->man.s_packed) ? 1u : 0u;
     const bool complete = !(pdl && !timing) && !c->ctrl->early_notify.load();
+    // A complete snapshot from one source: TMA bulk copies or register
+    // streaming with prefetched descriptors + seals (install_direct).
+    // VIPER_INSTALL_KERNEL=tma|direct|verify overrides the automatic choice (A/B).
+    static const char *ik = getenv("VIPER_INSTALL_KERNEL");
+    const bool tma_auto = ik ? strcmp(ik, "tma") == 0 : kInstallTmaDefault && c->man.s_packed <= (1ull << 30);
     const bool tma = direct && complete && !(c->cfg.flags & VIPER_FLAG_NO_TMA) &&
-                     ((c->cfg.flags & VIPER_FLAG_TMA) || c->man.s_packed <= (1ull << 30));
+                     ((c->cfg.flags & VIPER_FLAG_TMA) || tma_auto);
+    const bool use_direct = direct && complete && !tma && !(ik && strcmp(ik, "verify") == 0);
+    int launch_dev = c->device;
+    cudaGetDevice(&launch_dev);  // a SYNC publish launches on the producer's GPU
+    pi.a.sys_swap = launch_dev != c->device ? 1u : 0u;
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
     if (pdl && !timing && !tma) CUDA_TRY(launch_install(pi.a, c->geo, st, true));  // PDL: a plain stream launch
-    else CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms), pi.a, st));
+    else CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms, use_direct),
+                              pi.a, st));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
         c->timing_pending = true;
@@ -476,6 +507,58 @@ viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
     return st;
 }
 
+// The producer of a cross-process channel still exists (its pid in Ctrl).
+static bool producer_alive(const viper_model *c) {
+    if (!c->xproc) return true;
+    if (c->ctrl->closing.load()) return false;
+    const int32_t pid = c->ctrl->prod_pid.load();
+    return pid <= 0 || !(kill(pid, 0) == -1 && errno == ESRCH);
+}
+
+// Wait for the install enqueued on c->ustream, bounded: poll the
+// stream instead of blocking in cudaStreamSynchronize, and give up when the
+// consumer is unregistering, the producer process is gone or 60 s passed.  A
+// DRAM-tier install may sit in cuStreamWaitValue64 on a piece flag that a dead
+// producer never raises: giving up releases those flags from the host and
+// tells the kernel (rec->abort) to stop waiting for seals, so the stream
+// drains and the install reports VIPER_E_PEER / VIPER_E_TIMEOUT.
+static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
+    const int64_t t0 = now_ns();
+    if (getenv("VIPER_DEBUG")) fprintf(stderr, "[viper] waiting for the install of v%llu (slot %d)\n", (unsigned long long)v, b);
+    for (uint32_t spins = 0;; spins++) {
+        const cudaError_t e = cudaStreamQuery(c->ustream);
+        if (e == cudaSuccess) return VIPER_OK;
+        if (e != cudaErrorNotReady) return set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
+        const int64_t dt = now_ns() - t0;
+        if ((spins & 255) == 255) {
+            viper_status why = VIPER_OK;
+            if (c->stop.load()) why = set_error(VIPER_E_STATE, "install of v%llu abandoned: unregistering",
+                                                (unsigned long long)v);
+            else if (!producer_alive(c)) why = set_error(VIPER_E_PEER, "producer gone during the install of v%llu",
+                                                         (unsigned long long)v);
+            else if (dt > 60ll * 1000000000ll) why = set_error(VIPER_E_TIMEOUT, "install of v%llu did not finish in 60 s",
+                                                             (unsigned long long)v);
+            if (why != VIPER_OK) {
+                static const bool dbg = getenv("VIPER_DEBUG") != nullptr;
+                if (dbg) fprintf(stderr, "[viper] install of v%llu abandoned: %s\n", (unsigned long long)v, viper_last_error());
+                c->rec->abort.store(1);
+                if (c->cfg.tier == VIPER_TIER_DRAM)  // release the copy stream's flag waits
+                    for (size_t i = 0; i < c->man.piece_lo.size(); i++) {
+                        uint64_t cur = c->ctrl->dram_flag[b][i].load();
+                        while (cur < v && !c->ctrl->dram_flag[b][i].compare_exchange_weak(cur, v)) {
+                        }
+                    }
+                const cudaError_t se = cudaStreamSynchronize(c->ustream);  // bounded now: the kernel stops waiting
+                if (dbg) fprintf(stderr, "[viper] drained after abort: %s\n", cudaGetErrorString(se));
+                c->rec->abort.store(0);
+                return why;
+            }
+        }
+        if (dt < 200000) cpu_relax();
+        else usleep(dt < 10000000 ? 20 : 200);
+    }
+}
+
 void update_loop(viper_model *c) {
     cudaSetDevice(c->device);
     Ctrl *ctrl = c->ctrl;
@@ -528,8 +611,11 @@ void update_loop(viper_model *c) {
         const int64_t t0 = now_ns();
         NvtxRange nvtx("viper_install");
         viper_status st;
+        static const bool dbg = getenv("VIPER_DEBUG") != nullptr;
+        if (dbg) fprintf(stderr, "[viper] update thread: installing v%llu from slot %d\n", (unsigned long long)v, b);
         if (c->xproc) {
             st = xproc_install(c, v, b);
+            if (dbg) fprintf(stderr, "[viper] update thread: enqueued v%llu: %d %s\n", (unsigned long long)v, st, t_err.c_str());
         } else {
             // install_mu is held through the stream sync below: a producer
             // teardown drains this before freeing the buffers read here
@@ -537,10 +623,7 @@ void update_loop(viper_model *c) {
             st = p ? enqueue_install(c, source_of(p), v, b, c->ustream, true)
                    : set_error(VIPER_E_STATE, "producer gone");
         }
-        if (st == VIPER_OK) {
-            cudaError_t e = cudaStreamSynchronize(c->ustream);
-            if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
-        }
+        if (st == VIPER_OK) st = wait_install_bounded(c, v, b);
         if (st == VIPER_OK) st = finish_install(c, v, (now_ns() - t0) / 1e3);
         else {
             r->status.store(st);
@@ -691,7 +774,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     // PDL-chained to (profiles/r01: faster up to ~1 GB, slightly slower above)
     const bool tma_auto = !(p->cfg.flags & VIPER_FLAG_NO_TMA) && (!sync || dram || p->xproc) &&
                           p->man.s_packed <= (1ull << 30);
-    const bool tma = ((p->cfg.flags & VIPER_FLAG_TMA) || tma_auto) && !p->early_notify;
+    const bool tma = ((p->cfg.flags & VIPER_FLAG_TMA) || tma_auto) && !p->early_notify && !staged_fanout(p->cfg.fanout);
     const bool fuse = sync && !dram && !prepared.empty() && prepared.size() <= (size_t)kMaxFused &&
                       !(p->cfg.flags & (VIPER_FLAG_NO_FUSE | VIPER_FLAG_TMA));
     if (fuse) {
@@ -707,6 +790,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         for (size_t k = 0; k < prepared.size(); k++) {
             const InstallArgs &ia = prepared[k].a;
             f.cons[k] = FusedCons{ia.items, ia.target, ia.fault_item, ia.status_h, ia.pin_h, ia.state_h};
+            if (prepared[k].c->device != p->device) f.sys_swap = 1;
             prepared[k].c->rec->status.store(1);
             std::lock_guard<std::mutex> lk(prepared[k].c->stats_mu);
             prepared[k].c->stats.writer_wait_us = prepared[k].waited_us;
@@ -734,8 +818,30 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // a PDL-chained install must follow a plain stream launch; every
         // other pack goes through its one-node graph (cheaper on the host)
         const bool pdl_follows = sync && !dram && !tma && !prepared.empty();
-        if (pdl_follows) CUDA_TRY(launch_pack(a, p->geo, st));
-        else if (a.nitems) CUDA_TRY(launch_spec(p->g_pack, pack_launch(a, p->geo, tma, p->device), a, st));
+        if (p->cfg.fanout == VIPER_FANOUT_PUSH && a.nitems) {
+            // push: the same pack also stores every item into each consumer's staging
+            PushArgs pa{};
+            pa.p = a;
+            pa.ndst = (uint32_t)p->npush;
+            for (int k = 0; k < p->npush; k++) {
+                pa.dst[k] = p->push_dst[b][k];
+                pa.dst_iseal[k] = p->push_iseal[b][k];
+            }
+            CUDA_TRY(launch_spec(p->g_pack, push_launch(p->geo), pa, st));
+        } else if (p->cfg.fanout == VIPER_FANOUT_NVLS && a.nitems) {
+            // NVLS: one store per vector to the multicast address (snapshot + every consumer)
+            NvlsArgs na{};
+            na.items = a.items;
+            na.nitems = a.nitems;
+            na.mc_packed = p->nvls_mc_snap[b];
+            na.mc_iseal = p->nvls_mc_iseal[b];
+            na.version = v;
+            CUDA_TRY(launch_spec(p->g_pack, nvls_launch(p->geo), na, st));
+        } else if (pdl_follows) {
+            CUDA_TRY(launch_pack(a, p->geo, st));
+        } else if (a.nitems) {
+            CUDA_TRY(launch_spec(p->g_pack, pack_launch(a, p->geo, tma, p->device), a, st));
+        }
         if (timing) {
             CUDA_TRY(cudaEventRecord(p->ev_t[1], st));
             p->timing_pending = true;
@@ -792,6 +898,10 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
             if (i + 1 == np)  // item seals once, before the last flag (one copy instead of one per piece)
                 CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b], p->d_iseal[b], sizeof(ISeal) * mm.items.size(),
                                          cudaMemcpyDeviceToHost, p->side));
+            // VIPER_TEST_DRAM_STALL=1 (tests): never raise the flags, as a
+            // producer that died mid-transfer would not
+            static const bool stall = getenv("VIPER_TEST_DRAM_STALL") && atoi(getenv("VIPER_TEST_DRAM_STALL"));
+            if (stall) continue;
             viper_status s = stream_write(p->side, &p->ctrl_dev->dram_flag[b][i], v);
             if (s) return s;
         }
@@ -976,7 +1086,7 @@ viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
         if ((st = upload_items(m->man, m->slot_ptrs[s], &m->d_slot_items[s], 1, 0, nullptr))) return st;
     CUDA_TRY(cudaMalloc(&m->d_flags, 64));
     CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
-    if (m->cfg.tier == VIPER_TIER_DRAM) {
+    if (m->cfg.tier == VIPER_TIER_DRAM || m->cfg.fanout == VIPER_FANOUT_CE) {
         const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
         CUDA_TRY(cudaMalloc(&m->stage_alloc, al256(S) + IS));
         m->d_stage = (uint8_t *)m->stage_alloc;
@@ -1056,13 +1166,29 @@ static viper_status register_local(viper_model *m, const viper_tensor *tensors) 
         std::lock_guard<std::mutex> lk(m->chan->mu);
         if (viper_model *p = channel_producer(m->chan))
             if ((st = link_devices(p->device, m->device, m->cfg.tier))) return st;
-        const int idx = m->ctrl->ncons.load();
-        if (idx >= kMaxConsumers) return set_error(VIPER_E_INVAL, "more than %d consumers", kMaxConsumers);
+        // reuse the record of a consumer that unregistered (no reader left on
+        // it), so restarting consumers never exhaust the kMaxConsumers records;
+        // ncons stays the high-water mark the scans cover
+        int idx = -1;
+        const int n = m->ctrl->ncons.load();
+        for (int i = 0; i < n && idx < 0; i++) {
+            ConsRec &r = m->ctrl->cons[i];
+            if (!r.active.load() && r.ref[0].load() == 0 && r.ref[1].load() == 0) idx = i;
+        }
+        if (idx < 0 && n >= kMaxConsumers)
+            return set_error(VIPER_E_INVAL, "more than %d live consumers", kMaxConsumers);
+        if (idx < 0) idx = n;
         m->cidx = idx;
         m->rec = &m->ctrl->cons[idx];
         m->rec_dev = &m->ctrl_dev->cons[idx];
+        m->rec->state.store(0);
+        m->rec->pin.store(0);
+        m->rec->status.store(0);
+        m->rec->done_version.store(0);
+        m->rec->last_status.store(0);
+        m->rec->abort.store(0);
         m->rec->active.store(1);
-        m->ctrl->ncons.store(idx + 1);
+        if (idx == n) m->ctrl->ncons.store(idx + 1);
         m->chan->consumers.push_back(m);
     }
     m->upd = std::thread(update_loop, m);
@@ -1116,14 +1242,21 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
             return set_error(VIPER_E_INVAL, "bad tier");
         if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
         if (c.install_sms < 0) return set_error(VIPER_E_INVAL, "install_sms must be >= 0");
+        if (c.fanout == VIPER_FANOUT_NCCL)
+            return set_error(VIPER_E_UNSUPPORTED, "fanout NCCL is a bench.py baseline (torch.distributed.broadcast), "
+                                                  "not an engine transport");
         if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_CHAIN &&
-            c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER)
+            c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER && !xproc_only_fanout(c.fanout))
             return set_error(VIPER_E_UNSUPPORTED, "fanout %d not supported", c.fanout);
+        if (xproc_only_fanout(c.fanout) && !(bs && bs->world > 1))
+            return set_error(VIPER_E_UNSUPPORTED, "fanout %d (NVLS / push / CE) needs the cross-process channel",
+                             c.fanout);
         int ndev = 0;
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0)
             return set_error(VIPER_E_CUDA, "no CUDA device (there is no CPU fallback)");
         if (c.device < 0 || c.device >= ndev) return set_error(VIPER_E_INVAL, "bad device %d", c.device);
         CUDA_TRY(cudaSetDevice(c.device));
+        CUDA_TRY(preload_kernels());
         st = check_tensor_devices(tensors, n, c.device);
         if (st) return st;
         viper_model *m = new viper_model();
@@ -1328,6 +1461,28 @@ viper_status viper_debug_buffers(viper_model *m, void **dev_packed, void **dev_s
         if (dev_packed) *dev_packed = m->d_stage;
         if (dev_seals) *dev_seals = nullptr;
     }
+    return VIPER_OK;
+}
+
+viper_status viper_view_seals(viper_model *m, const viper_view *view, void *dev_seals_out, void *cuda_stream) {
+    if (!m || !view || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
+    if (m->role != VIPER_CONSUMER) return set_error(VIPER_E_STATE, "view_seals on a producer");
+    if (!dev_seals_out && m->man.nchunks) return set_error(VIPER_E_INVAL, "dev_seals_out is NULL");
+    {
+        std::lock_guard<std::mutex> lk(m->views_mu);
+        auto it = m->views.find(view->ticket);
+        if (it == m->views.end() || it->second.slot != view->slot)
+            return set_error(VIPER_E_STATE, "unknown or released view (ticket %llu)", (unsigned long long)view->ticket);
+    }
+    CUDA_TRY(cudaSetDevice(m->device));
+    const cudaStream_t st = (cudaStream_t)cuda_stream;
+    if (m->man.nchunks) CUDA_TRY(cudaMemsetAsync(dev_seals_out, 0, sizeof(Seal) * m->man.nchunks, st));
+    ViewSealArgs a{};
+    a.items = m->d_slot_items[view->slot];
+    a.nitems = (uint32_t)m->man.items.size();
+    a.seals = (Seal *)dev_seals_out;
+    a.version = view->version;
+    CUDA_TRY(launch_view_seals(a, st));
     return VIPER_OK;
 }
 

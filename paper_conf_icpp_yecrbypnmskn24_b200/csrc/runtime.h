@@ -30,6 +30,14 @@ constexpr int kMaxPieces = 256;     // DRAM tier: D2H / H2D pipeline granularity
 constexpr int kMaxProducers = 8;   // data-parallel producers (multi-producer fan-in)
 constexpr uint64_t kCtrlMagic = 0x5649504552435431ull;  // "VIPERCT1"
 
+// Fan-outs that exist only across processes (one producer, GPU tier).
+inline bool xproc_only_fanout(int32_t f) {
+    return f == VIPER_FANOUT_NVLS || f == VIPER_FANOUT_PUSH || f == VIPER_FANOUT_CE;
+}
+// Consumers install from a local staging buffer the producer writes into
+// (push: peer stores; NVLS: multicast stores).
+inline bool staged_fanout(int32_t f) { return f == VIPER_FANOUT_NVLS || f == VIPER_FANOUT_PUSH; }
+
 struct alignas(64) ConsRec {
     std::atomic<uint64_t> state;         // (v << 1) | slot, 0 = nothing installed (device-written)
     std::atomic<uint64_t> pin;           // snapshot version being read, 0 = none (device-cleared)
@@ -43,6 +51,8 @@ struct alignas(64) ConsRec {
     std::atomic<int32_t> pid;            // consumer process (failure detection), 0 = in-process
     std::atomic<uint64_t> p1_done;       // scatter-allgather: phase-1 version finished
     std::atomic<uint64_t> p2_done;       // scatter-allgather: phase-2 version finished
+    std::atomic<int32_t> abort;          // host -> install kernel: stop waiting for item seals (the
+                                         // update thread gave up: producer gone, unregister, deadline)
 };
 
 struct alignas(64) Ctrl {
@@ -62,6 +72,7 @@ struct alignas(64) Ctrl {
     alignas(64) std::atomic<uint64_t> pub_m[kMaxProducers];
     std::atomic<int32_t> nprod;
     std::atomic<int32_t> early_notify;   // producer names v before its pack completed
+    std::atomic<int32_t> prod_pid;       // cross-process producer (liveness), 0 = in-process
 };
 
 // Pointer-free work item (the device lists add each endpoint's tensor address).
@@ -199,6 +210,20 @@ struct viper_model {
     uint32_t pack_nitems = 0;                        // items this producer packs (its chunk share)
     void *peer_snap_m[vp::kMaxProducers] = {};        // consumer: every producer's snapshot (IPC)
     void *d_mp_tab = nullptr;                        // consumer: snap[2][M], iseal[2][M]
+    // push / NVLS (staged fan-outs): consumers install from their own staging
+    vp::SnapSource stage_src;                        // consumer: staging slot b + its item seals
+    void *push_peer_base[vp::kMaxPush] = {};         // producer (push): consumers' staging (IPC-opened)
+    uint8_t *push_dst[2][vp::kMaxPush] = {};         // producer (push): consumer k's staging slot b
+    vp::ISeal *push_iseal[2][vp::kMaxPush] = {};
+    int32_t npush = 0;
+    // NVLS (nvls.cpp): one multicast object; driver handles kept as integers
+    uint64_t nvls_mc = 0, nvls_phys = 0, nvls_va = 0, nvls_uc = 0;
+    size_t nvls_bytes = 0;
+    int nvls_fd = -1, nvls_listen = -1;
+    bool nvls_have_mc = false, nvls_have_phys = false, nvls_bound = false, nvls_uc_mapped = false,
+         nvls_mc_mapped = false;
+    uint8_t *nvls_mc_snap[2] = {nullptr, nullptr};   // producer: multicast VA of snapshot slot b
+    vp::ISeal *nvls_mc_iseal[2] = {nullptr, nullptr};
 
     // ---------------- stats
     std::mutex stats_mu;
@@ -268,5 +293,13 @@ viper_status xproc_notify(viper_model *p, uint64_t v, int b, bool sync, bool alr
 viper_status xproc_notify_early(viper_model *p, uint64_t v, int b, cudaStream_t st);           // producer
 void xproc_abort(const viper_bootstrap *bs, viper_status st);  // failed before the bootstrap
 void xproc_free(viper_model *m);
+
+// nvls.cpp (VIPER_FANOUT_NVLS); every failure is VIPER_E_UNSUPPORTED / _PEER
+viper_status nvls_probe(int device);
+viper_status nvls_create(viper_model *m, int nranks, size_t bytes, char *sock_name, size_t cap);  // producer
+viper_status nvls_serve(viper_model *m, int nconsumers);                                          // producer
+viper_status nvls_join(viper_model *m, const char *sock_name, size_t bytes);                      // consumer
+viper_status nvls_bind(viper_model *m, bool map_mc);                                              // every rank
+void nvls_free(viper_model *m);
 
 }  // namespace vp

@@ -55,6 +55,26 @@ struct PackArgs {
                                 // (set when the snapshot fits in L2, so it stays there)
 };
 
+// Push delivery (VIPER_FANOUT_PUSH): the pack also stores every item into
+// each consumer's peer-mapped staging slot and releases its seal there.
+constexpr int kMaxPush = 8;
+struct PushArgs {
+    PackArgs p;                 // the local pack (snapshot + item seals)
+    uint32_t ndst;              // consumers
+    uint8_t *dst[kMaxPush];     // consumer k's staging for this snapshot slot (peer-mapped)
+    ISeal *dst_iseal[kMaxPush]; // consumer k's staging item seals
+};
+
+// NVLS multicast delivery (VIPER_FANOUT_NVLS): stores go to the multicast
+// address of the snapshot slot; NVSwitch replicates them to every bound rank.
+struct NvlsArgs {
+    const Item *items;
+    uint32_t nitems;
+    uint8_t *mc_packed;         // multicast VA of snapshot slot b
+    ISeal *mc_iseal;            // multicast VA of its item seals
+    uint64_t version;
+};
+
 struct SealReduceArgs {
     const uint32_t *chunk_first;  // [nchunks + 1] item ranges of the chunks
     uint32_t nchunks;
@@ -63,6 +83,17 @@ struct SealReduceArgs {
     uint64_t version;
     uint32_t share_n, share_me;   // multi-producer: only chunks c % share_n == share_me
 };
+
+// viper_view_seals: chunk seals of a consumer slot, computed in place.
+struct ViewSealArgs {
+    const Item *items;          // the slot's work list (ptr = slot tensor piece)
+    uint32_t nitems;
+    Seal *seals;                // [nchunks], zeroed by the caller; {version, cks} (written)
+    uint64_t version;
+};
+cudaError_t launch_view_seals(const ViewSealArgs &a, cudaStream_t st);
+// load every kernel into the current device's context (no lazy load at a launch)
+cudaError_t preload_kernels();
 
 struct InstallArgs {
     const Item *items;          // consumer list of the target slot (ptr = slot tensor piece)
@@ -80,6 +111,7 @@ struct InstallArgs {
     volatile int32_t *status_h;
     volatile uint64_t *pin_h;
     volatile uint64_t *state_h;
+    const volatile int32_t *abort_h;  // host-mapped: nonzero = stop waiting for seals (report a timeout)
     // Scatter-allgather fan-out (sa_n > 0): item x is owned by consumer
     // chunk(x) % sa_n.  Owned items come from the producer (`packed`) and are
     // also written to this consumer's staging (+ seal, release.sys) for its
@@ -101,6 +133,7 @@ struct InstallArgs {
     const ISeal *const *sa_isrc;                 // [sa_n] peers' staging seals
     const volatile uint64_t *const *sa_owner_pin;  // [sa_n] peers' pin words (host-mapped)
     uint32_t l2_once;           // TMA variant: load the snapshot with an L2 evict-first hint
+    uint32_t sys_swap;          // the slot is on another GPU than the kernel: system-scope fence before the swap
 };
 
 // SYNC in-process publish (K2+K6 fused): each warp packs its item,
@@ -125,6 +158,7 @@ struct FusedArgs {
     unsigned long long *flags;  // [1] low 32: blocks finished; high 32: bit k = consumer k failed (self-resetting);
                                 // flags + 1: the work counter (kernels.cu WorkQueue), reset by the last block
     FusedCons cons[kMaxFused];
+    uint32_t sys_swap;          // a consumer slot is on another GPU: system-scope fence before the swaps
 };
 
 struct Geometry {
@@ -156,8 +190,18 @@ FusedLaunch fused_tma_launch(uint32_t nitems, int device);
 // pack_seal (register, geometry g) or pack_seal_tma; seal_reduce
 LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int device);
 LaunchSpec seal_reduce_launch(const SealReduceArgs &a);
-// install_verify (register, geometry g, not PDL-chained) or install_verify_tma
-LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms);
+// pack_push / pack_nvls (register streaming, geometry g)
+LaunchSpec push_launch(const Geometry &g);
+LaunchSpec nvls_launch(const Geometry &g);
+// install_verify (register, geometry g, not PDL-chained), install_verify_tma, or
+// install_direct (direct = a complete snapshot from one source, register streaming)
+LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms,
+                          bool direct = false);
+#ifndef VP_INSTALL_TMA_DEFAULT
+#define VP_INSTALL_TMA_DEFAULT 1
+#endif
+// complete-snapshot installs <= 1 GiB use the TMA kernel (else install_direct)
+constexpr bool kInstallTmaDefault = VP_INSTALL_TMA_DEFAULT != 0;
 #ifndef VP_FUSED_TMA_DEFAULT
 #define VP_FUSED_TMA_DEFAULT 0
 #endif

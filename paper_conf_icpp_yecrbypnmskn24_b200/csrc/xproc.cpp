@@ -47,6 +47,8 @@ struct PeerRec {
     cudaIpcMemHandle_t sa_handle;            // consumer staging (scatter-allgather)
     int32_t cidx;
     char pci[32];                            // PCI bus id of the rank's GPU
+    char nvls_sock[64];                      // producer, NVLS: abstract socket serving the multicast fd
+    uint64_t nvls_bytes;                     // producer, NVLS: size of the multicast object
 };
 
 uint64_t fnv1a(const void *p, size_t n, uint64_t h = 0xcbf29ce484222325ull) {
@@ -282,6 +284,14 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank/nproducers", bs->rank);
     if (st == VIPER_OK && M > 1 && (m->cfg.tier != VIPER_TIER_GPU || m->cfg.fanout != VIPER_FANOUT_DIRECT))
         st = set_error(VIPER_E_UNSUPPORTED, "data-parallel producers: GPU tier, direct fan-out only");
+    const bool nvls = m->cfg.fanout == VIPER_FANOUT_NVLS;
+    const bool push = m->cfg.fanout == VIPER_FANOUT_PUSH;
+    if (st == VIPER_OK && xproc_only_fanout(m->cfg.fanout) && m->cfg.tier != VIPER_TIER_GPU)
+        st = set_error(VIPER_E_UNSUPPORTED, "fan-out %d needs the GPU tier (the Transfer Selector chose DRAM)",
+                       m->cfg.fanout);
+    if (st == VIPER_OK && push && bs->world - M > kMaxPush)
+        st = set_error(VIPER_E_UNSUPPORTED, "push fan-out: at most %d consumers", kMaxPush);
+    if (st == VIPER_OK && nvls && !producer) st = nvls_probe(m->device);  // reported in allgather #1
     const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
     const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
     const size_t ctrl_bytes = page_up(sizeof(Ctrl));
@@ -298,6 +308,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             c->magic = kCtrlMagic;
             c->ncons.store(bs->world - M);
             c->nprod.store(M);
+            c->prod_pid.store((int32_t)getpid());
             st = map_control(m);
         }
         if (st == VIPER_OK) {
@@ -316,11 +327,15 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             const cudaError_t e = cudaIpcGetMemHandle(&me.snap_handle, m->snap_alloc);
             if (e != cudaSuccess) st = set_error(VIPER_E_CUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
         }
+        if (st == VIPER_OK && nvls) {  // the multicast object: snapshot + item seals, both slots
+            st = nvls_create(m, bs->world, 2 * (S + IS), me.nvls_sock, sizeof me.nvls_sock);
+            me.nvls_bytes = m->nvls_bytes;
+        }
     }
     // consumers stage what their peers pull from them: the chunks they own
     // (scatter-allgather) or everything (chain)
     const bool sa = m->cfg.fanout == VIPER_FANOUT_SCATTER_ALLGATHER || m->cfg.fanout == VIPER_FANOUT_CHAIN;
-    if (st == VIPER_OK && !producer && sa) {
+    if (st == VIPER_OK && !producer && (sa || push)) {  // push: the producer stores into this staging
         // my staging, double-buffered by snapshot slot
         m->sa_S = S;
         m->sa_IS = IS;
@@ -338,12 +353,73 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
     if (st == VIPER_OK) {
         for (int r = 0; r < bs->world; r++) {
             if (all[r].magic != kPeerMagic) st = set_error(VIPER_E_PEER, "rank %d sent a bad record", r);
+            else if (all[r].status == VIPER_E_UNSUPPORTED)  // e.g. no multicast on that GPU: same answer everywhere
+                st = set_error(VIPER_E_UNSUPPORTED, "rank %d: fan-out %d unsupported there", r, m->cfg.fanout);
             else if (all[r].status != VIPER_OK) st = set_error(VIPER_E_PEER, "rank %d failed to register", r);
             else if (all[r].manifest_hash != me.manifest_hash)
                 st = set_error(VIPER_E_INVAL, "rank %d registered a different tensor list", r);
             else if (all[r].tier != me.tier || all[r].fanout != me.fanout)
                 st = set_error(VIPER_E_INVAL, "rank %d uses another tier / fan-out", r);
         }
+    }
+    if (st == VIPER_OK && nvls) {  // NVLS binds one buffer per GPU: ranks must not share a GPU
+        for (int r = 0; r < bs->world && st == VIPER_OK; r++)
+            for (int q = r + 1; q < bs->world; q++)
+                if (strncmp(all[r].pci, all[q].pci, sizeof me.pci) == 0) {
+                    st = set_error(VIPER_E_UNSUPPORTED, "NVLS: ranks %d and %d share GPU %s", r, q, all[r].pci);
+                    break;
+                }
+    }
+    if (st == VIPER_OK && nvls) st = producer ? nvls_serve(m, bs->world - M) : nvls_join(m, pr.nvls_sock, pr.nvls_bytes);
+    {
+        // allgather #1b (every rank, every fan-out, so the rounds always match):
+        // every GPU joined the multicast object before anyone binds memory
+        PeerRec mid{};
+        mid.magic = kPeerMagic;
+        mid.status = st;
+        std::vector<PeerRec> ms(bs->world);
+        if (bs->allgather(&mid, ms.data(), sizeof(PeerRec), bs->user) != 0)
+            return set_error(VIPER_E_PEER, "bootstrap allgather #1b failed");
+        for (int r = 0; r < bs->world && st == VIPER_OK; r++)
+            if (ms[r].status != VIPER_OK)
+                st = set_error(ms[r].status == VIPER_E_UNSUPPORTED ? VIPER_E_UNSUPPORTED : VIPER_E_PEER,
+                               "rank %d failed to register", r);
+    }
+    if (st == VIPER_OK && nvls) {
+        st = nvls_bind(m, producer);
+        if (st == VIPER_OK) {
+            uint8_t *uc = (uint8_t *)m->nvls_uc;
+            for (int b = 0; b < 2; b++) {
+                ISeal *is = (ISeal *)(uc + 2 * S + b * IS);
+                if (producer) {  // the snapshot IS this GPU's share of the multicast object
+                    m->d_snap[b] = uc + b * S;
+                    m->d_iseal[b] = is;
+                    m->nvls_mc_snap[b] = (uint8_t *)m->nvls_va + b * S;
+                    m->nvls_mc_iseal[b] = (ISeal *)((uint8_t *)m->nvls_va + 2 * S + b * IS);
+                } else {
+                    m->stage_src.snap[b] = uc + b * S;
+                    m->stage_src.iseal[b] = is;
+                }
+            }
+        }
+    }
+    if (st == VIPER_OK && producer && push) {  // map every consumer's staging
+        int k = 0;
+        for (int r = 0; r < bs->world && st == VIPER_OK; r++) {
+            if (all[r].role == VIPER_PRODUCER) continue;
+            const cudaError_t e =
+                cudaIpcOpenMemHandle(&m->push_peer_base[k], all[r].sa_handle, cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess) {
+                st = set_error(VIPER_E_PEER, "push: cudaIpcOpenMemHandle (rank %d): %s", r, cudaGetErrorString(e));
+                break;
+            }
+            for (int b = 0; b < 2; b++) {
+                m->push_dst[b][k] = (uint8_t *)m->push_peer_base[k] + b * S;
+                m->push_iseal[b][k] = (ISeal *)((uint8_t *)m->push_peer_base[k] + 2 * S + b * IS);
+            }
+            k++;
+        }
+        m->npush = k;
     }
     if (st == VIPER_OK && producer && m->pidx > 0) {  // data-parallel producer j > 0: join the segment
         st = open_segment(m, pr.shm_path, pr.shm_bytes);
@@ -357,6 +433,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (all[r].role != VIPER_PRODUCER && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
         const char *env = getenv("VIPER_EARLY_NOTIFY");
         m->early_notify = env ? atoi(env) != 0 : other;
+        if (m->cfg.fanout == VIPER_FANOUT_CE) m->early_notify = false;  // the copy engine needs a sealed snapshot
         if (m->pidx == 0) m->ctrl->early_notify.store(m->early_notify ? 1 : 0);
     }
     if (st == VIPER_OK && !producer) {
@@ -388,6 +465,12 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             st = alloc_consumer(m, tensors);
         }
         if (st == VIPER_OK && sa) st = open_sa_peers(m, all, bs);
+        if (st == VIPER_OK && push) {  // install from the staging the producer pushes into
+            for (int b = 0; b < 2; b++) {
+                m->stage_src.snap[b] = (const uint8_t *)m->sa_alloc + b * S;
+                m->stage_src.iseal[b] = (const ISeal *)((const uint8_t *)m->sa_alloc + 2 * S + b * IS);
+            }
+        }
         if (st == VIPER_OK && M > 1) st = open_producers(m, all, bs);
         if (st == VIPER_OK) {
             m->rec->pid.store((int32_t)getpid());
@@ -403,7 +486,9 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         return set_error(VIPER_E_PEER, "bootstrap allgather #2 failed");
     if (st != VIPER_OK) return st;
     for (int r = 0; r < bs->world; r++)
-        if (sts[r].status != VIPER_OK) return set_error(VIPER_E_PEER, "rank %d failed to register", r);
+        if (sts[r].status != VIPER_OK)
+            return set_error(sts[r].status == VIPER_E_UNSUPPORTED ? VIPER_E_UNSUPPORTED : VIPER_E_PEER,
+                             "rank %d failed to register", r);
     if (!producer) m->upd = std::thread(update_loop, m);
     return VIPER_OK;
 }
@@ -419,8 +504,9 @@ void xproc_abort(const viper_bootstrap *bs, viper_status st) {
     me.rank = bs->rank;
     me.status = st;
     std::vector<PeerRec> all(bs->world > 0 ? bs->world : 1);
-    if (bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user) != 0) return;
-    bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user);
+    // allgathers #1, #1b and #2 of xproc_register
+    for (int round = 0; round < 3; round++)
+        if (bs->allgather(&me, all.data(), sizeof(PeerRec), bs->user) != 0) return;
 }
 
 // Consumer update thread (install_mu held, v pinned): pull slot b of the
@@ -437,6 +523,8 @@ viper_status xproc_install(viper_model *c, uint64_t v, int b) {
         pi.a.mp_iseal = (const ISeal *const *)(tab + 2 * M + b * M);
         return launch_prepared(pi, c->xsrc, b, c->ustream, false, false);
     }
+    if (staged_fanout(c->cfg.fanout))  // push / NVLS: the producer wrote into this GPU's staging
+        return enqueue_install(c, c->stage_src, v, b, c->ustream, false);
     const bool chain = c->cfg.fanout == VIPER_FANOUT_CHAIN;
     if ((c->cfg.fanout != VIPER_FANOUT_SCATTER_ALLGATHER && !chain) || c->nconsumers_x < 2 ||
         c->cfg.tier != VIPER_TIER_GPU)
@@ -537,6 +625,9 @@ void xproc_free(viper_model *m) {
         if (p) cudaIpcCloseMemHandle(p), p = nullptr;
     for (auto &p : m->peer_snap_m)
         if (p) cudaIpcCloseMemHandle(p), p = nullptr;
+    for (auto &p : m->push_peer_base)
+        if (p) cudaIpcCloseMemHandle(p), p = nullptr;
+    nvls_free(m);
     cudaFree(m->d_mp_tab);
     m->d_mp_tab = nullptr;
     cudaFree(m->d_sa_tab);

@@ -17,7 +17,8 @@ OK, E_INVAL, E_NOMEM, E_CUDA, E_VERSION, E_CHECKSUM, E_TIMEOUT, E_NOVERSION, E_S
 PRODUCER, CONSUMER = 1, 2
 F32, BF16, F16, BYTES = 0, 1, 2, 3
 TIER_GPU, TIER_DRAM, TIER_AUTO = 0, 1, 2
-FANOUT_DIRECT, FANOUT_CHAIN, FANOUT_SCATTER_ALLGATHER = 0, 1, 2
+FANOUT_DIRECT, FANOUT_CHAIN, FANOUT_SCATTER_ALLGATHER, FANOUT_NVLS, FANOUT_PUSH = 0, 1, 2, 3, 4
+FANOUT_NCCL, FANOUT_CE = 100, 101  # baselines (include/viper.h)
 SYNC, ASYNC = 0, 1
 FLAG_TIMING = 2
 FLAG_NO_FUSE = 4
@@ -81,6 +82,7 @@ UPDATE_CB = C.CFUNCTYPE(None, C.c_uint64, C.c_int32, C.c_void_p)
 # every symbol include/viper.h declares (checked by tests/test_abi.py)
 EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_acquire_latest", "viper_release",
            "viper_wait_installed", "viper_get_stats", "viper_layout", "viper_debug_buffers", "viper_debug_fault_next", "viper_unregister",
+           "viper_view_seals",
            "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version",
            "viper_debug_proto_create", "viper_debug_proto_open", "viper_debug_proto_close",
            "viper_debug_proto_publish", "viper_debug_proto_install", "viper_debug_proto_read",
@@ -122,6 +124,7 @@ def lib() -> C.CDLL:
             L.viper_debug_buffers.argtypes = [C.c_void_p, C.POINTER(C.c_void_p), C.POINTER(C.c_void_p),
                                               C.POINTER(C.c_uint64)]
             L.viper_debug_fault_next.argtypes = [C.c_void_p]
+            L.viper_view_seals.argtypes = [C.c_void_p, C.POINTER(viper_view), C.c_void_p, C.c_void_p]
             L.viper_unregister.argtypes = [C.c_void_p]
             L.viper_schedule.argtypes = [C.POINTER(viper_sched_in), C.POINTER(viper_sched_out)]
             L.viper_debug_proto_create.argtypes = [C.c_char_p, C.c_uint64, C.c_int32, C.POINTER(C.c_void_p)]
@@ -277,6 +280,12 @@ class Model:
 
     def wait_installed(self, version: int, timeout_us: int = 10_000_000):
         check(lib().viper_wait_installed(self.h, version, timeout_us), f"viper_wait_installed({version})")
+
+    def view_seals(self, view: View, out, stream=None):
+        """Chunk seals {version, cks} of a pinned view's slot into `out` (a CUDA
+        tensor of >= 16 * nchunks bytes), computed on the device."""
+        check(lib().viper_view_seals(self.h, C.byref(view.raw), C.c_void_p(out.data_ptr()), _stream_ptr(stream)),
+              "viper_view_seals")
 
     def fault_next(self):
         check(lib().viper_debug_fault_next(self.h), "viper_debug_fault_next")

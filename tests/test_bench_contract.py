@@ -30,3 +30,62 @@ def test_reference_arm_json_line():
         assert k in d, k
     assert d["impl"] == "reference" and d["higher_is_better"] is False and d["value"] > 0
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["cpu_baseline"]["kind"] == "oracle"
+
+
+def _json_lines(out):
+    return [json.loads(l) for l in out.splitlines() if l.strip().startswith("{")]
+
+
+def test_gpus_n_self_launches_ranks():
+    """`bench.py --gpus 2` without a launcher starts 2 ranks
+    itself (torch.distributed.run on 127.0.0.1); on this CPU box the ranks
+    rendezvous over gloo, reduce over ranks and rank 0 prints ONE line with
+    n_gpus = 2 and no number (there is no GPU to measure)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--oversubscribe", "--steps", "3", "--warmup", "3"],
+                       cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True, timeout=300, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = lines[0]
+    assert d["n_gpus"] == 2 and d["ranks_seen"] == 2 and d["value"] is None and "unavailable" in d
+
+
+def test_gpus_n_fails_loudly_without_gpus():
+    """--gpus 2 with fewer visible GPUs and no --oversubscribe: non-zero exit,
+    no JSON line (never a silent 1-GPU measurement)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--steps", "3"], cwd=ROOT, stdout=subprocess.PIPE,
+                       stderr=subprocess.PIPE, text=True, timeout=120, env=env)
+    assert r.returncode != 0 and not _json_lines(r.stdout)
+    assert "--oversubscribe" in r.stderr
+
+
+def test_gpus_must_match_world_size():
+    env = dict(os.environ, WORLD_SIZE="1", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, "bench.py", "--gpus", "2", "--steps", "3"], cwd=ROOT, stdout=subprocess.PIPE,
+                       stderr=subprocess.PIPE, text=True, timeout=120, env=env)
+    assert r.returncode != 0 and "WORLD_SIZE=1" in r.stderr
+
+
+def test_reference_arm_under_two_ranks():
+    """--impl reference at N = 2: rank 0 alone runs the oracle with the N = 2
+    config (1 -> 1); the other rank exits without work; one line."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--oversubscribe",
+                        "--steps", "3", "--warmup", "3", "--cpu-budget", "0.5"], cwd=ROOT, stdout=subprocess.PIPE,
+                       stderr=subprocess.PIPE, text=True, timeout=300, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1 and lines[0]["impl"] == "reference" and lines[0]["n_gpus"] == 2
+
+
+def test_cpu_baseline_p_threads():
+    """the oracle on 1 thread and on P threads (disjoint tensor
+    subsets), with the core count stated."""
+    import bench
+    import synth
+    cb = bench.cpu_baseline(synth, "ptychonn", budget_s=0.3, max_updates=5)
+    assert cb["cores"] == 1 and cb["kind"] == "oracle" and cb["value"] > 0
+    p = cb["p_threads"]
+    assert p["cores"] >= 1 and p["value"] > 0 and p["cores"] <= cb["cpu"]["affinity_cores"]

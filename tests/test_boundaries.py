@@ -61,7 +61,7 @@ def test_bench_uses_the_oracle_only_in_its_baseline_legs():
     top = {n.module for n in tree.body if isinstance(n, ast.ImportFrom) and n.module}
     top |= {a.name for n in tree.body if isinstance(n, ast.Import) for a in n.names}
     assert not any(m.startswith("oracle") for m in top)
-    importers, users = set(), set()
+    importers, users, par_users = set(), set(), set()
     scopes = [n for n in ast.walk(tree) if isinstance(n, (ast.FunctionDef, ast.ClassDef))]
     for sc in scopes:
         for node in ast.walk(sc):
@@ -72,5 +72,10 @@ def test_bench_uses_the_oracle_only_in_its_baseline_legs():
             if isinstance(sc, ast.FunctionDef) and isinstance(node, ast.Call) and \
                     getattr(node.func, "id", None) == "OracleUpdates":
                 users.add(sc.name)
+            if isinstance(sc, ast.FunctionDef) and isinstance(node, ast.Call) and \
+                    getattr(node.func, "id", None) == "oracle_parallel":
+                par_users.add(sc.name)
     assert importers <= {"OracleUpdates", "__init__"} and "OracleUpdates" in importers, importers
-    assert users and users <= {"cpu_baseline", "reference_arm"}, users
+    # oracle_parallel (the P-thread oracle baseline) is part of the cpu_baseline leg only
+    assert users and users <= {"cpu_baseline", "reference_arm", "oracle_parallel"}, users
+    assert par_users <= {"cpu_baseline"}, par_users

@@ -54,6 +54,15 @@ def device_packed_and_seals(prod):
     return host_bytes(packed), seals.cpu().numpy().view(np.uint64).reshape(n, 2)
 
 
+def view_seals_host(c, view):
+    """viper_view_seals: the installed slot's chunk seals, computed on the GPU."""
+    n = c.stats()["nchunks"]
+    buf = torch.empty(max(16 * n, 16), dtype=torch.uint8, device="cuda")
+    c.view_seals(view, buf)
+    torch.cuda.synchronize()
+    return buf.view(torch.int64).cpu().numpy().view(np.uint64).reshape(-1, 2)[:n]
+
+
 def check_slot(view, cons_like, specs, seed, v):
     got = view.tensors(cons_like)
     exp = expect(specs, seed, v)
@@ -136,6 +145,7 @@ def test_ragged_tensor_lists_many_chunks(seed):
                 view = c.acquire_latest()
                 assert view.version == v
                 check_slot(view, ct, specs, 77 + seed, v)
+                assert np.array_equal(view_seals_host(c, view), s_or)  # installed-slot seals == oracle
                 c.release(view)
     finally:
         close_all(prod, cons)
@@ -643,3 +653,88 @@ def test_example_train_and_serve():
     same, served = tas.main(steps=30, every=3, verbose=False)
     assert same
     assert served["n"] > 0 and len(served["versions"]) >= 2
+
+
+# ------------------------------------------------------------ round 2 additions
+def test_view_seals_unaligned_and_errors():
+    """viper_view_seals on byte-offset (unaligned) slot tensors == the oracle's
+    chunk seals; a released view or a producer is rejected (VIPER_E_STATE)."""
+    specs = [("a", synth.BYTES, (1001,)), ("b", synth.BYTES, (4099,)), ("c", synth.BYTES, (37,))]
+    base_p = torch.empty(6000, dtype=torch.uint8, device="cuda")
+    base_c = torch.empty(6000, dtype=torch.uint8, device="cuda")
+    prod_t = [base_p[1:1002], base_p[1003:5102], base_p[5103:5140]]
+    cons_t = [base_c[3:1004], base_c[1005:5104], base_c[5105:5142]]
+    name = uname()
+    cons = V.Model(name, V.CONSUMER, cons_t, chunk_bytes=1024)
+    prod = V.Model(name, V.PRODUCER, prod_t, chunk_bytes=1024)
+    try:
+        for v in (1, 2):
+            G.fill_model(prod_t, specs, 0xAB, v)
+            prod.publish(v)
+            view = cons.acquire_latest()
+            _, s_or, _ = oracle_packed_and_seals(specs, 0xAB, v, 1024)
+            assert np.array_equal(view_seals_host(cons, view), s_or)
+            cons.release(view)
+        buf = torch.empty(16 * 16, dtype=torch.uint8, device="cuda")
+        with pytest.raises(V.ViperError) as e:
+            cons.view_seals(view, buf)  # released
+        assert e.value.status == V.E_STATE
+    finally:
+        cons.close()
+        prod.close()
+
+
+@pytest.mark.parametrize("name", ["resnet50", "vit_b16"])
+def test_golden_seals_full_size_in_process(name):
+    """At BASELINE.json full size: VGEN(seed, VCHECK) published SYNC and ASYNC;
+    the snapshot's and the installed slot's chunk seals == the oracle-written
+    tests/golden/seals file, every chunk."""
+    specs = synth.model_specs(name)
+    hdr, gold = synth.golden_seals(name)
+    for mode in (V.SYNC, V.ASYNC):
+        prod, prod_t, cons, cons_t = make_pair(specs, synth.SEEDS[name], mode=mode)
+        try:
+            G.fill_model(prod_t, specs, synth.SEEDS[name], synth.VCHECK)
+            prod.publish(3)
+            cons[0].wait_installed(3)
+            _, s_dev = device_packed_and_seals(prod)
+            assert [int(x) for x in s_dev[:, 1]] == gold
+            view = cons[0].acquire_latest()
+            cs = view_seals_host(cons[0], view)
+            assert (cs[:, 0] == 3).all() and [int(x) for x in cs[:, 1]] == gold
+            cons[0].release(view)
+        finally:
+            close_all(prod, cons)
+
+
+@pytest.mark.parametrize("fanout", [V.FANOUT_NVLS, V.FANOUT_PUSH, V.FANOUT_CE, V.FANOUT_NCCL])
+def test_cross_process_only_fanouts_rejected_in_process(fanout):
+    specs = synth.model_specs("ptychonn")
+    t = G.alloc_model(specs)
+    with pytest.raises(V.ViperError) as e:
+        V.Model(uname(), V.PRODUCER, t, fanout=fanout)
+    assert e.value.status == V.E_UNSUPPORTED
+
+
+def test_consumer_records_are_reused():
+    """consumers that unregister free their control record, so
+    a long-lived producer serves more than kMaxConsumers (16) consumers over
+    its life; each new one installs the next version bit-exactly."""
+    specs = [("w", synth.F32, (4096,)), ("b", synth.F32, (7,))]
+    prod_t = G.alloc_model(specs)
+    name = uname()
+    prod = V.Model(name, V.PRODUCER, prod_t)
+    try:
+        for k in range(20):
+            ct = G.alloc_model(specs)
+            c = V.Model(name, V.CONSUMER, ct)
+            G.fill_model(prod_t, specs, 0x5E, k + 1)
+            prod.publish(k + 1)
+            view = c.acquire_latest()
+            assert view.version == k + 1
+            check_slot(view, ct, specs, 0x5E, k + 1)
+            c.release(view)
+            c.close()
+        assert prod.stats()["nconsumers"] <= 2
+    finally:
+        prod.close()

@@ -178,3 +178,66 @@ def test_protocol_two_processes_gloo_cpu():
     0 torn snapshot copies, 0 torn reads, no version regress over 3000 publishes."""
     rc, out = run_torchrun(2, "tests/protocol_worker.py", [], timeout=180)
     assert rc == 0 and "PROTO_RESULT errors=0" in out, out[-3000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,mode,config", [(2, 0, "ptychonn"), (3, 0, "small"), (4, 1, "small"),
+                                              (2, 0, "resnet50"), (5, 0, "resnet50")])
+def test_xproc_push(nproc, mode, config):
+    """VIPER_FANOUT_PUSH: the producer's pack stores every item into
+    each consumer's peer-mapped staging and releases its seal there; consumers
+    install from local memory.  Bit-exact slots and installed-slot seals ==
+    the oracle's, every version."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", config, "--mode", str(mode), "--fanout", "4", "--versions", "5"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,fanout", [(3, 4), (2, 4)])
+def test_xproc_push_early_notify(nproc, fanout):
+    """Push with the cross-GPU item pipeline forced on: consumers wait per item
+    on the seals the producer releases (system scope) into their staging."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", "resnet50", "--fanout", str(fanout), "--versions", "4"],
+                           env={"VIPER_EARLY_NOTIFY": "1"})
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc,mode,config", [(2, 0, "ptychonn"), (3, 1, "small"), (3, 0, "resnet50")])
+def test_xproc_copy_engine_fanout(nproc, mode, config):
+    """VIPER_FANOUT_CE (SURVEY B2 as an engine mode): consumers copy the sealed
+    snapshot with cudaMemcpyAsync, then install + verify locally."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", config, "--mode", str(mode), "--fanout", "101", "--versions", "4"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+def test_xproc_push_fault():
+    rc, out = run_torchrun(3, "tests/xproc_worker.py", ["--config", "small", "--fanout", "4", "--fault", "1",
+                                                       "--versions", "3"])
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("nproc", [2, 3])
+def test_xproc_nvls_bit_exact_or_unsupported_everywhere(nproc):
+    """VIPER_FANOUT_NVLS: bit-exact where the box exposes multicast (one GPU per
+    rank, fabric manager); otherwise EVERY rank's registration fails with
+    VIPER_E_UNSUPPORTED (a 1-GPU lease: ranks share a GPU) -- never a hang or a
+    mixed outcome."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", "resnet50", "--fanout", "3", "--versions", "4", "--allow-unsupported"])
+    assert rc == 0, out[-4000:]
+    assert "XPROC_RESULT errors=0" in out or "XPROC_UNSUPPORTED everywhere=True" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+def test_xproc_dram_install_does_not_hang_on_a_vanished_producer():
+    """a DRAM-tier consumer whose producer named v but never raised
+    the pieces' flags (VIPER_TEST_DRAM_STALL) gives the install up once the
+    producer unregisters: VIPER_E_PEER, v not installed, prompt unregister."""
+    rc, out = run_torchrun(2, "tests/xproc_stall_worker.py", [], timeout=120)
+    assert "STALL_CONSUMER" in out and "ok=True" in out, out[-4000:]

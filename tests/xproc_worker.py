@@ -86,6 +86,8 @@ def main():
                     "(VIPER_TIER_AUTO resolved by the Transfer Selector)")
     ap.add_argument("--no-peer-rank", type=int, default=-1, help="this rank reports that it reaches no GPU "
                     "(VIPER_TEST_NO_PEER)")
+    ap.add_argument("--allow-unsupported", action="store_true",
+                    help="registration may fail with VIPER_E_UNSUPPORTED on EVERY rank (NVLS without multicast)")
     a = ap.parse_args()
     dist.init_process_group("gloo")
     rank, world = dist.get_rank(), dist.get_world_size()
@@ -100,8 +102,17 @@ def main():
     role = V.PRODUCER if is_prod else V.CONSUMER
     if rank == a.no_peer_rank:
         os.environ["VIPER_TEST_NO_PEER"] = "1"
-    m = V.Model(f"xp-{a.config}", role, tensors, tier=a.tier, mode=a.mode, fanout=a.fanout, device=dev,
-                bootstrap=bs)
+    try:
+        m = V.Model(f"xp-{a.config}", role, tensors, tier=a.tier, mode=a.mode, fanout=a.fanout, device=dev,
+                    bootstrap=bs)
+    except V.ViperError as e:
+        unsupported = e.status == V.E_UNSUPPORTED
+        t = torch.tensor([0 if unsupported else 1])
+        dist.all_reduce(t)
+        if rank == 0:
+            print(f"XPROC_UNSUPPORTED everywhere={int(t.item()) == 0}: {e.detail}", flush=True)
+        dist.destroy_process_group()
+        sys.exit(0 if (a.allow_unsupported and int(t.item()) == 0) else 1)
     errors = 0
     if a.expect_tier >= 0 and m.stats()["tier"] != a.expect_tier:
         print(f"[rank{rank}] tier {m.stats()['tier']}, want {a.expect_tier}", flush=True)
@@ -147,11 +158,22 @@ def main():
                 errors += 1
             last = view.version
             got = view.tensors(tensors)
-            for i, (g, s) in enumerate(zip(got, specs)):
-                if not np.array_equal(host_bytes(g), synth.vgen_numpy(seed, view.version, i, s[1], synth.nelem_of(s))):
+            exp = [synth.vgen_numpy(seed, view.version, i, s[1], synth.nelem_of(s)) for i, s in enumerate(specs)]
+            for i, (g, e) in enumerate(zip(got, exp)):
+                if not np.array_equal(host_bytes(g), e):
                     print(f"[rank{rank}] tensor {i} differs at v{view.version}", flush=True)
                     errors += 1
                     break
+            # the installed slot's chunk seals, computed on this GPU, == the oracle's
+            n = m.stats()["nchunks"]
+            sb = torch.empty(max(16 * n, 16), dtype=torch.uint8, device=f"cuda:{dev}")
+            m.view_seals(view, sb)
+            torch.cuda.synchronize()
+            cs = sb.view(torch.int64).cpu().numpy().view(np.uint64).reshape(-1, 2)[:n]
+            off, S = T.layout([e.size for e in exp], 256)
+            if not np.array_equal(cs, T.seal(T.pack(exp, off, S), 2 << 20, view.version)):
+                print(f"[rank{rank}] installed-slot seals differ from the oracle at v{view.version}", flush=True)
+                errors += 1
             m.release(view)
         dist.barrier()
     if not is_prod and a.mode == V.ASYNC and not a.stress:

@@ -18,18 +18,22 @@ ap.add_argument("--flush", action="store_true")
 ap.add_argument("--tier", type=int, default=0)
 ap.add_argument("--nofuse", action="store_true")
 ap.add_argument("--flags", type=int, default=0, help="extra VIPER_FLAG_* bits for the producer")
+ap.add_argument("--cflags", type=int, default=0, help="VIPER_FLAG_* bits for the consumer")
+ap.add_argument("--mode", type=int, default=0, help="0 SYNC, 1 ASYNC (the consumer's update thread installs)")
 a = ap.parse_args()
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
 pt, ct = G.alloc_model(specs), G.alloc_model(specs)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if a.flush else None
-c = V.Model("prof", V.CONSUMER, ct, tier=a.tier)
-p = V.Model("prof", V.PRODUCER, pt, tier=a.tier, flags=(V.FLAG_NO_FUSE if a.nofuse else 0) | a.flags)
+c = V.Model("prof", V.CONSUMER, ct, tier=a.tier, flags=a.cflags)
+p = V.Model("prof", V.PRODUCER, pt, tier=a.tier, flags=(V.FLAG_NO_FUSE if a.nofuse else 0) | a.flags, mode=a.mode)
 for v in range(1, a.steps + 1):
     G.fill_model(pt, specs, seed, v)
     if flush is not None:
         G.l2_flush(flush)
     p.publish(v)
+    if a.mode == V.ASYNC:
+        c.wait_installed(v)
 torch.cuda.synchronize()
 c.close()
 p.close()
