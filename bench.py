@@ -68,7 +68,7 @@ def ncu_traffic(kernel, config):
         return None
 
 
-LAUNCH_LISTS = {"resnet50": "profiles/r01/launches_bench_r50_summary.json",
+LAUNCH_LISTS = {"resnet50": "profiles/r02/launches_bench_r50_summary.json",
                 "ptychonn": "profiles/r01/launches_bench_c1_summary.json"}
 
 
@@ -739,6 +739,11 @@ FANOUT_NAMES = {0: "direct pull", 1: "pipelined chain", 2: "scatter-allgather", 
 NVLINK_GBS = 900.0  # NVLink 5 per direction per GPU (north_star / B200_PROFILING.md)
 
 
+def log(msg):
+    """Progress of the N > 1 arm on stderr (rank-tagged; the JSON line stays alone on stdout)."""
+    print(f"[bench rank {os.environ.get('RANK', '0')} {time.strftime('%H:%M:%S')}] {msg}", file=sys.stderr, flush=True)
+
+
 def verify_replicas(V, G, synth, m, name, rank, tensors, dev):
     """Bit-exact evidence for one cross-process run, without the oracle at bench
     time: the LAST published version carries VGEN(seed, synth.VCHECK), whose
@@ -801,10 +806,12 @@ def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, step
     seed = synth.SEEDS[name]
     tensors = G.alloc_model(specs)
     bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
+    log(f"{name} fan-out {fanout}: registering")
     try:
         m = V.Model(f"bench-x-{name}-{fanout}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors, fanout=fanout,
                     flags=V.FLAG_TIMING if rank else 0, device=dev, bootstrap=bs)
     except V.ViperError as e:
+        log(f"fan-out {fanout}: {e.name}")
         del tensors
         torch.cuda.empty_cache()
         return {"unsupported": f"{e.name}: {e.detail}"[:300]}
@@ -832,6 +839,7 @@ def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, step
             dist.barrier(group=gloo)
             if rank != 0 and i >= warmup:
                 inst.append(m.stats()["t_install_dev_us"])
+        log(f"fan-out {fanout}: {steps} timed updates done; verification version")
         # verification version: the golden content
         if rank == 0:
             G.fill_model(tensors, specs, seed, synth.VCHECK)
@@ -843,8 +851,10 @@ def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, step
         dist.barrier(group=gloo)
         ver = verify_replicas(V, G, synth, m, name, rank, tensors, dev)
         ver["version_ok"] = ver["version"] == warmup + steps + 1
+        log(f"fan-out {fanout}: verified {ver}")
         s_packed = m.stats()["s_packed"]
     finally:
+        log(f"fan-out {fanout}: closing")
         dist.barrier(group=gloo)
         if rank != 0:  # consumers first: they read the producer's buffers
             m.close()
@@ -853,6 +863,7 @@ def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, step
             m.close()
         del tensors
         torch.cuda.empty_cache()
+        log(f"fan-out {fanout}: closed")
     return {"lat": lat, "host": host, "inst": inst, "verify": ver, "s_packed": s_packed}
 
 
@@ -937,6 +948,7 @@ def xproc_concurrent(V, G, synth, name, rank, world, dev, gloo, fanout, seconds=
                     cnt["views"] += 1
 
         for phase in ("idle", "busy"):
+            log(f"concurrent acquire: {phase}")
             dist.barrier(group=gloo)
             cnt["views"] = 0
             th = threading.Thread(target=reader) if rank else None
@@ -998,6 +1010,9 @@ def xproc_arm(args):
     import torch
     import torch.distributed as dist
     rank, world, local = dist_env()
+    if os.environ.get("BENCH_WATCHDOG_S"):  # debugging: dump every thread's Python stack if the arm stalls
+        import faulthandler
+        faulthandler.dump_traceback_later(int(os.environ["BENCH_WATCHDOG_S"]), repeat=True)
     if not torch.cuda.is_available() or torch.cuda.device_count() == 0:
         # no GPU (CPU plumbing check of the launcher): rendezvous, max over
         # ranks, one line from rank 0 -- and no number
@@ -1046,10 +1061,12 @@ def xproc_arm(args):
             if f == "push" and world - 1 > 8:
                 continue
             r = xproc_updates(V, G, synth, name, rank, world, dev, gloo, FANOUTS[f], flush, args.steps, args.warmup)
-            results[f] = summarize_fanout(gather_obj(r, gloo), S) if rank == 0 else None
+            per_rank = gather_obj(r, gloo)  # collective: every rank
+            results[f] = summarize_fanout(per_rank, S) if rank == 0 else None
             dist.barrier(group=gloo)
     head = next((f for f in order if rank != 0 or "unsupported" not in results[f]), order[0])
     head = gather_obj(head, gloo)[0]
+    log(f"fan-outs timed, headline {head}; baselines")
     # baselines on the same bytes: NCCL broadcast (device time, max over ranks) and a torch copy-engine pull
     buf = torch.empty(S, dtype=torch.uint8, device="cuda")
     nccl_ms = []
@@ -1066,8 +1083,10 @@ def xproc_arm(args):
     ce_ms = ce_baseline(rank, gloo, buf, args.steps, args.warmup)
     del buf
     torch.cuda.empty_cache()
+    log("concurrent acquire")
     conc = xproc_concurrent(V, G, synth, name, rank, world, dev, gloo, FANOUTS[head])
     conc_all = gather_obj(conc, gloo)
+    log("e2e")
     e2e = xproc_e2e(V, G, synth, name, rank, world, dev, gloo, FANOUTS[head], flush, args.steps, args.warmup)
     t = torch.tensor([statistics.mean(nccl_ms) if nccl_ms else 0.0, ce_ms, e2e["ms"], float(1 - e2e["ok"])],
                      dtype=torch.float64)

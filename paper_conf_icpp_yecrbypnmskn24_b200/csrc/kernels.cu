@@ -65,6 +65,21 @@ __device__ __forceinline__ uint4 ld_stream(const void *p) {
     return r;
 }
 
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+
+// The same with an L2 cache policy (createpolicy): read-once data evicted first
+__device__ __forceinline__ uint4 ld_stream_pol(const void *p, uint64_t pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p), "l"(pol));
+    return r;
+}
+
 __device__ __forceinline__ uint4 ld_cg(const void *p) {  // L2-coherent (data written during this grid)
     uint4 r;
     asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -167,9 +182,10 @@ __device__ __forceinline__ uint64_t copy_words_bytewise(const uint8_t *__restric
 
 // Copy one work item (src -> dst, n bytes, packed offset p0); returns the
 // lane's partial checksum of the packed-space words it moved.
+// pol != 0 (non-coherent loads only): L2 cache policy of the source loads
 template <bool kCoherent, int U = kUnroll>
 __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst, uint32_t n,
-                                              uint64_t p0, uint32_t lane, bool inject) {
+                                              uint64_t p0, uint32_t lane, bool inject, uint64_t pol = 0) {
     uint64_t acc = 0;
     const bool aligned = (((uintptr_t)src | (uintptr_t)dst) & 15u) == 0;
     if (!aligned) return copy_words_bytewise<kCoherent>(src, dst, 0, n, p0, lane, inject);
@@ -180,7 +196,9 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
 #pragma unroll
         for (int u = 0; u < U; u++) {
             const uint32_t i = base + u * 32 + lane;
-            if (i < nvec) r[u] = kCoherent ? ld_cg(src + (size_t)i * 16) : ld_stream(src + (size_t)i * 16);
+            if (i < nvec)
+                r[u] = kCoherent ? ld_cg(src + (size_t)i * 16)
+                                 : (pol ? ld_stream_pol(src + (size_t)i * 16, pol) : ld_stream(src + (size_t)i * 16));
         }
         if (inject && base == 0 && lane == 0) r[0].x ^= 0x10u;
 #pragma unroll
@@ -698,72 +716,90 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
     install_finish(a, bad);
 }
 
-// install_direct: the install of a COMPLETE snapshot (nothing left to wait
-// for: not PDL-chained, not early-notified) from one source -- the local or
+// install_direct: the install of one version from ONE source -- the local or
 // NVLink-peer-mapped snapshot, or this GPU's staging (push / NVLS / CE / DRAM
-// tier).  The pack's structure: static item striding, and the next item's
-// descriptor AND its seal {cks, version} fetched one item ahead, so a warp's
-// only dependent round trip per item is its data.  The source is immutable
-// for the grid's lifetime (the consumer pins it), so the data is read with
-// non-coherent streaming loads.  A seal that does not show `version` yet (it
-// cannot, for a complete snapshot, but the kernel never trusts that) falls
-// back to the acquire spin of install_verify_kernel.
+// tier) -- with the pack's structure: static item striding, and the next
+// item's descriptor fetched one item ahead.
+//   kPipe = false: the snapshot is COMPLETE before the grid starts (not
+//     PDL-chained, not early-notified).  The next item's seal {cks, version}
+//     is fetched one item ahead too, so a warp's only dependent round trip per
+//     item is its data, and the data is immutable for the grid's lifetime (the
+//     consumer pins it): non-coherent streaming loads.  A seal that does not
+//     show `version` (it cannot, but the kernel never trusts that) falls back
+//     to the acquire spin.
+//   kPipe = true: the item pipeline behind a pack that is still running
+//     (PDL on this GPU, early notification across GPUs): lane 0 acquires the
+//     item's seal at system scope before the warp streams it, with
+//     L2-coherent loads.  Only direct installs; scatter-allgather / chain /
+//     data-parallel producers keep install_verify_kernel.
+// U = 16-B vectors per lane in flight: 16 for snapshots <= 1 GiB, 8 above
+// (ncu cold sweep, profiles/r02/install_sweep.json).
 __device__ __forceinline__ ISeal ld_seal(const ISeal *p) {
     ISeal s;
     asm volatile("ld.global.cg.v2.u64 {%0,%1}, [%2];" : "=l"(s.mixed), "=l"(s.version) : "l"(p));
     return s;
 }
 
-#ifndef VP_ID_UNROLL
-#define VP_ID_UNROLL 8
-#endif
 #ifndef VP_ID_BLOCKS
 #define VP_ID_BLOCKS 2
 #endif
-constexpr int kIdUnroll = VP_ID_UNROLL;  // install_direct's own geometry (sweep: profiles/r02)
-constexpr int kIdBlocks = VP_ID_BLOCKS;
+constexpr int kIdBlocks = VP_ID_BLOCKS;  // install_direct's resident blocks per SM
 
+// lane 0: wait until item w's seal shows the version (acquire, system scope:
+// the producer may be another GPU); returns its cks.  Never hangs.
+__device__ __forceinline__ uint64_t acquire_seal(const InstallArgs &a, uint32_t w) {
+    uint32_t backoff = 32;
+    uint64_t waited = 0;
+    while (ld_acquire_sys(&a.iseal[w].version) != a.version) {
+        __nanosleep(backoff);
+        waited += backoff;
+        if (backoff < 1024) backoff <<= 1;
+        if (waited > kItemWaitNs || wait_aborted(a)) {
+            report_err(a.flags, kErrTimeout);
+            break;
+        }
+    }
+    return a.iseal[w].mixed;
+}
+
+template <int U, bool kPipe>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kIdBlocks) install_direct_kernel(const InstallArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     bool bad = false;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    // a snapshot that fits in L2 was usually just written there: read it with
+    // an evict-first policy so the slot stores do not push out the lines not
+    // read yet (as the TMA install does, profiles/r01/tma_l2_hint_ab.log)
+    const uint64_t pol = (!kPipe && a.l2_once) ? l2_evict_first_policy() : 0;
     Item nxt{};
     ISeal nseal{};
     if (w < a.nitems) {
         nxt = a.items[w];
-        if (lane == 0) nseal = ld_seal(a.iseal + w);
+        if (!kPipe && lane == 0) nseal = ld_seal(a.iseal + w);
     }
     for (; w < a.nitems; w += nwarps) {
         const Item it = nxt;
         uint64_t expect = 0;
-        if (lane == 0) {
-            if (nseal.version != a.version) {  // not expected for a complete snapshot: wait like install_verify
-                uint32_t backoff = 32;
-                uint64_t waited = 0;
-                while (ld_acquire_sys(&a.iseal[w].version) != a.version) {
-                    __nanosleep(backoff);
-                    waited += backoff;
-                    if (backoff < 1024) backoff <<= 1;
-                    if (waited > kItemWaitNs || wait_aborted(a)) {
-                        report_err(a.flags, kErrTimeout);
-                        break;
-                    }
-                }
-                nseal.mixed = a.iseal[w].mixed;
-            }
-            expect = nseal.mixed;
-        }
+        if (lane == 0) expect = (kPipe || nseal.version != a.version) ? acquire_seal(a, w) : nseal.mixed;
+        if (kPipe) __syncwarp();  // the data loads below follow lane 0's acquire
         const uint32_t wn = w + nwarps;  // prefetch: its loads overlap this item's stream
         if (wn < a.nitems) {
             nxt = a.items[wn];
-            if (lane == 0) nseal = ld_seal(a.iseal + wn);
+            if (!kPipe && lane == 0) nseal = ld_seal(a.iseal + wn);
         }
-        const uint64_t part = warp_sum(copy_item<false, kIdUnroll>(a.packed + it.packed_off, (uint8_t *)it.ptr,
-                                                                   it.nbytes, it.packed_off, lane, w == a.fault_item));
+        const uint64_t part = warp_sum(copy_item<kPipe, U>(a.packed + it.packed_off, (uint8_t *)it.ptr, it.nbytes,
+                                                           it.packed_off, lane, w == a.fault_item, pol));
         if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
     }
     install_finish(a, bad);
+}
+
+// the instantiation for a snapshot of `bytes`
+static const void *install_direct_fn(uint64_t bytes, bool pipe) {
+    const bool big = bytes > (1ull << 30);
+    if (pipe) return big ? (const void *)install_direct_kernel<8, true> : (const void *)install_direct_kernel<16, true>;
+    return big ? (const void *)install_direct_kernel<8, false> : (const void *)install_direct_kernel<16, false>;
 }
 
 // SYNC in-process publish, pack + install fused per warp.  Lane l re-reads
@@ -896,11 +932,6 @@ __device__ __forceinline__ void bulk_g2s(void *smem, const void *gmem, uint32_t 
 // L2 policy for data read exactly once (the pack's parameter tensors, the
 // install's snapshot): evict it first, so it does not push out data that is
 // read again soon (the snapshot the install or the D2H reads next).
-__device__ __forceinline__ uint64_t l2_evict_first_policy() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-    return pol;
-}
 
 // pol == 0: no hint (models larger than L2 gain nothing from it and lose a little)
 __device__ __forceinline__ void bulk_g2s_once(void *smem, const void *gmem, uint32_t bytes, uint64_t *bar,
@@ -1477,11 +1508,12 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
     return l;
 }
 
-LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms, bool direct) {
+LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms, bool direct,
+                          uint64_t s_packed, bool pipe) {
     LaunchSpec l{};
     if (direct && !tma) {
         const int sms = sm_count(launch_device());
-        l.func = (const void *)install_direct_kernel;
+        l.func = install_direct_fn(s_packed, pipe);
         l.grid = grid_for(a.nitems, kWarpsPerBlock, max_sms > 0 && max_sms < sms ? max_sms : sms, kIdBlocks);
         l.block = g.block;
     } else if (tma) {
@@ -1542,7 +1574,9 @@ cudaError_t preload_kernels() {
     const uint64_t bit = 1ull << (dev >= 0 && dev < kMaxDevices ? dev : 0);
     if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
     const void *fns[] = {(const void *)pack_seal_kernel,         (const void *)seal_reduce_kernel,
-                         (const void *)install_verify_kernel,    (const void *)install_direct_kernel,
+                         (const void *)install_verify_kernel,    install_direct_fn(0, false),
+                         install_direct_fn(~0ull, false),        install_direct_fn(0, true),
+                         install_direct_fn(~0ull, true),
                          (const void *)publish_fused_kernel,     (const void *)pack_seal_tma_kernel,
                          (const void *)install_verify_tma_kernel, (const void *)publish_fused_tma_kernel,
                          (const void *)view_seal_kernel,         (const void *)pack_push_kernel,
@@ -1573,7 +1607,8 @@ cudaError_t launch_view_seals(const ViewSealArgs &a, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl) {
+cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl, bool direct,
+                           uint64_t s_packed) {
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(g.grid);
     cfg.blockDim = dim3(g.block);
@@ -1583,7 +1618,11 @@ cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t
     attr[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = attr;
     cfg.numAttrs = pdl ? 1 : 0;
-    return cudaLaunchKernelEx(&cfg, install_verify_kernel, a);
+    if (!direct) return cudaLaunchKernelEx(&cfg, install_verify_kernel, a);
+    const int sms = sm_count(launch_device());
+    cfg.gridDim = dim3(grid_for(a.nitems, kWarpsPerBlock, sms, kIdBlocks));
+    void *args[] = {(void *)&a};
+    return cudaLaunchKernelExC(&cfg, install_direct_fn(s_packed, true), args);
 }
 
 }  // namespace vp

@@ -439,14 +439,20 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     const bool tma_auto = ik ? strcmp(ik, "tma") == 0 : kInstallTmaDefault && c->man.s_packed <= (1ull << 30);
     const bool tma = direct && complete && !(c->cfg.flags & VIPER_FLAG_NO_TMA) &&
                      ((c->cfg.flags & VIPER_FLAG_TMA) || tma_auto);
-    const bool use_direct = direct && complete && !tma && !(ik && strcmp(ik, "verify") == 0);
+    // install_direct for every one-source install, complete or pipelined (the
+    // old install_verify_kernel stays for fan-outs among consumers and
+    // data-parallel producers, and as the A/B: VIPER_INSTALL_KERNEL=verify)
+    const bool use_direct = direct && !tma && !(ik && strcmp(ik, "verify") == 0);
     int launch_dev = c->device;
     cudaGetDevice(&launch_dev);  // a SYNC publish launches on the producer's GPU
     pi.a.sys_swap = launch_dev != c->device ? 1u : 0u;
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
-    if (pdl && !timing && !tma) CUDA_TRY(launch_install(pi.a, c->geo, st, true));  // PDL: a plain stream launch
-    else CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms, use_direct),
-                              pi.a, st));
+    if (pdl && !timing && !tma)  // PDL: a plain stream launch
+        CUDA_TRY(launch_install(pi.a, c->geo, st, true, use_direct, c->man.s_packed));
+    else
+        CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms, use_direct,
+                                                       c->man.s_packed, !complete),
+                             pi.a, st));
     if (timing) {
         CUDA_TRY(cudaEventRecord(c->ev_t[1], st));
         c->timing_pending = true;
@@ -524,7 +530,8 @@ static bool producer_alive(const viper_model *c) {
 // drains and the install reports VIPER_E_PEER / VIPER_E_TIMEOUT.
 static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
     const int64_t t0 = now_ns();
-    if (getenv("VIPER_DEBUG")) fprintf(stderr, "[viper] waiting for the install of v%llu (slot %d)\n", (unsigned long long)v, b);
+    static const bool dbg_wait = getenv("VIPER_DEBUG") != nullptr;
+    if (dbg_wait) fprintf(stderr, "[viper] waiting for the install of v%llu (slot %d)\n", (unsigned long long)v, b);
     for (uint32_t spins = 0;; spins++) {
         const cudaError_t e = cudaStreamQuery(c->ustream);
         if (e == cudaSuccess) return VIPER_OK;
@@ -551,6 +558,10 @@ static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
                 const cudaError_t se = cudaStreamSynchronize(c->ustream);  // bounded now: the kernel stops waiting
                 if (dbg) fprintf(stderr, "[viper] drained after abort: %s\n", cudaGetErrorString(se));
                 c->rec->abort.store(0);
+                // the data may still have arrived complete (its seals verified
+                // every item and the kernel swapped): then v IS installed
+                if (se == cudaSuccess && c->rec->status.load() == VIPER_OK && (c->rec->state.load() >> 1) == v)
+                    return VIPER_OK;
                 return why;
             }
         }
@@ -892,16 +903,15 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         // raises its flag for the consumers' H2D
         const Manifest &mm = p->man;
         const size_t np = mm.piece_lo.size();
-        for (size_t i = 0; i < np; i++) {
+        // VIPER_TEST_DRAM_STALL=1 (tests): the producer named v but never
+        // delivers it (no copy, no flag), as one that died mid-transfer
+        static const bool stall = getenv("VIPER_TEST_DRAM_STALL") && atoi(getenv("VIPER_TEST_DRAM_STALL"));
+        for (size_t i = 0; i < np && !stall; i++) {
             CUDA_TRY(cudaMemcpyAsync(p->h_stage[b] + mm.piece_lo[i], p->d_snap[b] + mm.piece_lo[i],
                                      mm.piece_hi[i] - mm.piece_lo[i], cudaMemcpyDeviceToHost, p->side));
             if (i + 1 == np)  // item seals once, before the last flag (one copy instead of one per piece)
                 CUDA_TRY(cudaMemcpyAsync(p->h_iseal[b], p->d_iseal[b], sizeof(ISeal) * mm.items.size(),
                                          cudaMemcpyDeviceToHost, p->side));
-            // VIPER_TEST_DRAM_STALL=1 (tests): never raise the flags, as a
-            // producer that died mid-transfer would not
-            static const bool stall = getenv("VIPER_TEST_DRAM_STALL") && atoi(getenv("VIPER_TEST_DRAM_STALL"));
-            if (stall) continue;
             viper_status s = stream_write(p->side, &p->ctrl_dev->dram_flag[b][i], v);
             if (s) return s;
         }

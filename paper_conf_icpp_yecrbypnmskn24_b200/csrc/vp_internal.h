@@ -196,11 +196,14 @@ LaunchSpec nvls_launch(const Geometry &g);
 // install_verify (register, geometry g, not PDL-chained), install_verify_tma, or
 // install_direct (direct = a complete snapshot from one source, register streaming)
 LaunchSpec install_launch(const InstallArgs &a, const Geometry &g, bool tma, int device, int max_sms,
-                          bool direct = false);
+                          bool direct = false, uint64_t s_packed = 0, bool pipe = false);
 #ifndef VP_INSTALL_TMA_DEFAULT
 #define VP_INSTALL_TMA_DEFAULT 1
 #endif
-// complete-snapshot installs <= 1 GiB use the TMA kernel (else install_direct)
+// complete-snapshot installs <= 1 GiB use the TMA kernel (else install_direct).  Cold (ncu) the two tie
+// within 3%; right behind the pack that wrote the snapshot into L2 (CUDA events), TMA's asynchronous bulk
+// stores ride out the write-back of the dirty snapshot better: ResNet-50 34.2 vs 38.3 us
+// (profiles/r02/install_sweep.json, profiles/r02/ktime_install_ab.log)
 constexpr bool kInstallTmaDefault = VP_INSTALL_TMA_DEFAULT != 0;
 #ifndef VP_FUSED_TMA_DEFAULT
 #define VP_FUSED_TMA_DEFAULT 0
@@ -208,7 +211,9 @@ constexpr bool kInstallTmaDefault = VP_INSTALL_TMA_DEFAULT != 0;
 // SYNC in-process publishes use the TMA fused kernel (VIPER_FUSED_TMA=0/1 overrides)
 constexpr bool kFusedTmaDefault = VP_FUSED_TMA_DEFAULT != 0;
 constexpr uint64_t kFusedTmaMaxBytes = 1ull << 30;  // auto-selection limit (packed bytes)
-// pdl: the install directly follows the pack on `st` (programmatic dependent launch)
-cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl);
+// pdl: the install directly follows the pack on `st` (programmatic dependent launch);
+// direct: one source (install_direct_kernel, pipelined), else install_verify_kernel
+cudaError_t launch_install(const InstallArgs &a, const Geometry &g, cudaStream_t st, bool pdl, bool direct = false,
+                           uint64_t s_packed = 0);
 
 }  // namespace vp

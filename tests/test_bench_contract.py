@@ -89,3 +89,26 @@ def test_cpu_baseline_p_threads():
     assert cb["cores"] == 1 and cb["kind"] == "oracle" and cb["value"] > 0
     p = cb["p_threads"]
     assert p["cores"] >= 1 and p["value"] > 0 and p["cores"] <= cb["cpu"]["affinity_cores"]
+
+
+def test_summarize_fanout_math_and_parity():
+    """The N > 1 line's per-fan-out summary: value = max over ranks of the
+    device windows, f_NVL = S / L / 900 GB/s, parity requires every consumer's
+    golden-seal match, byte match and final version; an unsupported fan-out
+    (NVLS without multicast) is reported as such."""
+    import bench
+    S = 102228128
+    ver_ok = {"seals_ok": True, "bytes_ok": True, "chunks": 49, "version": 9, "version_ok": True}
+    prod = {"lat": [0.2, 0.2, 0.2], "host": [0.21] * 3, "inst": [], "verify": dict(ver_ok, bytes_ok=None),
+            "s_packed": S}
+    cons = {"lat": [], "host": [], "inst": [150.0, 160.0, 170.0], "verify": ver_ok, "s_packed": S}
+    r = bench.summarize_fanout([prod, cons], S)
+    assert abs(r["latency_ms"] - 0.2) < 1e-12
+    assert abs(r["nvlink_frac"] - S / 0.2e-3 / 1e9 / 900.0) < 1e-4
+    assert r["install_kernel_us_per_consumer"] == [160.0] and r["parity_ok"] is True
+    slow = dict(cons, inst=[300.0] * 3)  # a consumer whose install window exceeds the producer's
+    assert abs(bench.summarize_fanout([prod, slow], S)["latency_ms"] - 0.3) < 1e-12
+    bad = dict(cons, verify=dict(ver_ok, seals_ok=False))
+    assert bench.summarize_fanout([prod, bad], S)["parity_ok"] is False
+    un = bench.summarize_fanout([{"unsupported": "VIPER_E_UNSUPPORTED: no multicast"}] * 2, S)
+    assert "unsupported" in un

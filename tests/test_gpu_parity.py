@@ -738,3 +738,40 @@ def test_consumer_records_are_reused():
         assert prod.stats()["nconsumers"] <= 2
     finally:
         prod.close()
+
+
+@pytest.mark.skipif(torch.cuda.device_count() < 2, reason="needs two GPUs (in-process cross-device update)")
+@pytest.mark.parametrize("mode,flags", [(V.SYNC, 0), (V.SYNC, V.FLAG_NO_FUSE), (V.SYNC, V.FLAG_TMA),
+                                        (V.ASYNC, 0)])
+def test_two_gpus_in_process(mode, flags):
+    """producer on cuda:0, consumer on cuda:1 in one process.  SYNC
+    installs run on the producer's stream and write the peer slot (the TMA
+    install's shared-memory opt-in and the grid size are keyed on the
+    launching GPU; the swap is fenced at system scope); ASYNC installs run on
+    the consumer's GPU and pull the peer snapshot.  Bit-exact slots and
+    installed-slot seals == the oracle's."""
+    specs = synth.model_specs("resnet50")
+    seed = synth.SEEDS["resnet50"]
+    prod_t = G.alloc_model(specs, device="cuda:0")
+    cons_t = G.alloc_model(specs, device="cuda:1")
+    name = uname()
+    cons = V.Model(name, V.CONSUMER, cons_t, device=1)
+    prod = V.Model(name, V.PRODUCER, prod_t, device=0, mode=mode, flags=flags)
+    try:
+        for v in (1, 2, 3):
+            G.fill_model(prod_t, specs, seed, v)
+            prod.publish(v)
+            cons.wait_installed(v)
+            view = cons.acquire_latest()
+            assert view.version == v
+            check_slot(view, cons_t, specs, seed, v)
+            n = cons.stats()["nchunks"]
+            buf = torch.empty(16 * n, dtype=torch.uint8, device="cuda:1")
+            cons.view_seals(view, buf)
+            torch.cuda.synchronize(1)
+            _, s_or, _ = oracle_packed_and_seals(specs, seed, v, 2 << 20)
+            assert np.array_equal(buf.view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2), s_or)
+            cons.release(view)
+    finally:
+        cons.close()
+        prod.close()

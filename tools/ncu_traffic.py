@@ -10,9 +10,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def main(summary):
     d = json.load(open(summary))
-    out = {}
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    out = json.load(open(path)) if os.path.exists(path) else {}  # merge: newer captures replace their rows
     for rep, kernels in d.items():
-        cfg = rep.replace(".ncu-rep", "").split("_", 2)[-1]  # full_fused_<cfg> / full_sep_<cfg>
+        cfg = rep.replace(".ncu-rep", "").split("_")[-1]  # ..._<cfg>
+        cfg = {"r50": "resnet50", "vit": "vit_b16", "gpt2": "gpt2_xl"}.get(cfg, cfg)
         for k in kernels:
             name = k["kernel"].split("::")[-1].split("(")[0]
             rd, wr = k["dram__bytes_read.sum"], k["dram__bytes_write.sum"]
@@ -21,7 +23,7 @@ def main(summary):
                                     "grid": k.get("launch__grid_size"), "block": k.get("launch__block_size"),
                                     "registers": k.get("launch__registers_per_thread"),
                                     "source": f"{os.path.relpath(summary, ROOT)} ({rep})"}
-    with open(os.path.join(ROOT, "profiles", "ncu_traffic.json"), "w") as f:
+    with open(path, "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps(out, indent=1))
 
