@@ -733,9 +733,12 @@ def xproc_e2e(V, G, synth, name, rank, world, dev, group, fanout, flush_buf, ste
     return {"ms": statistics.mean(times) if times else 0.0, "h2d": flat.numel(), "d2h": 16 * nchunks, "ok": ok}
 
 
-FANOUTS = {"direct": 0, "chain": 1, "sa": 2, "nvls": 3, "push": 4, "ce": 101}  # include/viper.h VIPER_FANOUT_*
+# include/viper.h VIPER_FANOUT_*; "dram" (-1) = the pinned-DRAM tier (BASELINE configs[4]: DRAM-to-DRAM
+# staging vs direct GPU-to-GPU), direct fan-out
+FANOUTS = {"direct": 0, "chain": 1, "sa": 2, "nvls": 3, "push": 4, "ce": 101, "dram": -1}
 FANOUT_NAMES = {0: "direct pull", 1: "pipelined chain", 2: "scatter-allgather", 3: "NVLS multicast",
-                4: "push (producer stores into peer staging)", 101: "copy engine (engine baseline)"}
+                4: "push (producer stores into peer staging)", 101: "copy engine (engine baseline)",
+                -1: "pinned-DRAM tier (D2H -> shared host staging -> H2D)"}
 NVLINK_GBS = 900.0  # NVLink 5 per direction per GPU (north_star / B200_PROFILING.md)
 
 
@@ -807,9 +810,10 @@ def xproc_updates(V, G, synth, name, rank, world, dev, gloo, fanout, flush, step
     tensors = G.alloc_model(specs)
     bs = V.Bootstrap(rank, world, producer_rank=0, group=gloo)
     log(f"{name} fan-out {fanout}: registering")
+    tier = V.TIER_DRAM if fanout == FANOUTS["dram"] else V.TIER_GPU
     try:
-        m = V.Model(f"bench-x-{name}-{fanout}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors, fanout=fanout,
-                    flags=V.FLAG_TIMING if rank else 0, device=dev, bootstrap=bs)
+        m = V.Model(f"bench-x-{name}-{fanout}", V.PRODUCER if rank == 0 else V.CONSUMER, tensors,
+                    fanout=max(fanout, 0), tier=tier, flags=V.FLAG_TIMING if rank else 0, device=dev, bootstrap=bs)
     except V.ViperError as e:
         log(f"fan-out {fanout}: {e.name}")
         del tensors
@@ -1050,11 +1054,11 @@ def xproc_arm(args):
     if args.fanout != "auto":
         order = [args.fanout]
     elif world == 2:
-        order = ["direct", "push", "ce", "nvls"]
+        order = ["direct", "push", "ce", "nvls", "dram"]
     else:
-        order = ["nvls", "sa", "chain", "push", "direct", "ce"]
+        order = ["nvls", "sa", "chain", "push", "direct", "ce", "dram"]
     if over and args.fanout == "auto":  # ranks time-slice one GPU: peer waits only serialise
-        order = ["direct", "push", "ce"]
+        order = ["direct", "push", "ce", "dram"]
     results = {}
     with ClockSampler(dev) as clk:
         for f in order:
@@ -1064,7 +1068,7 @@ def xproc_arm(args):
             per_rank = gather_obj(r, gloo)  # collective: every rank
             results[f] = summarize_fanout(per_rank, S) if rank == 0 else None
             dist.barrier(group=gloo)
-    head = next((f for f in order if rank != 0 or "unsupported" not in results[f]), order[0])
+    head = next((f for f in order if f != "dram" and (rank != 0 or "unsupported" not in results[f])), order[0])
     head = gather_obj(head, gloo)[0]
     log(f"fan-outs timed, headline {head}; baselines")
     # baselines on the same bytes: NCCL broadcast (device time, max over ranks) and a torch copy-engine pull
@@ -1120,6 +1124,10 @@ def xproc_arm(args):
                 "install_kernel": {"us": inst, "achieved": round(S / (inst * 1e-6) / 1e9, 2) if inst else None,
                                    "frac": h["install_kernel_nvlink_frac"]}},
             "fanouts": results,
+            "dram_over_gpu": (round(results["dram"]["latency_ms"] / lat_ms, 3)
+                              if ok and "latency_ms" in results.get("dram", {}) else None),
+            "dram_over_gpu_how": "BASELINE configs[4]: the pinned-DRAM tier's update latency over the headline "
+                                 "GPU-to-GPU fan-out, same bytes (paper context: TC1 Host-Async / GPU-Async 2.7x)",
             "parity_ok": h.get("parity_ok", False),
             "parity": h.get("parity"),
             "nccl_broadcast_ms": None if over else round(float(t[0]), 6),

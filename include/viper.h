@@ -353,6 +353,16 @@ viper_status viper_debug_proto_read(void *h, int32_t cidx, uint64_t *version, ui
 viper_status viper_debug_resolve_tier(const void *records, int32_t world, int32_t producer_rank,
                                       int32_t nproducers, int32_t fanout, int32_t requested, int32_t *out);
 
+/* Test hooks: the descriptor hand-off of NVLS registration (VIPER_FANOUT_NVLS),
+ * with no CUDA: an abstract Unix socket and SCM_RIGHTS.  listen: a fresh name
+ * (written to name_out, >= 32 bytes) and a listening socket; serve: hand `fd`
+ * to `n` fetchers, waiting at most timeout_ms for each (VIPER_E_PEER when one
+ * never connects), then close the socket; fetch: connect to `name` (retrying
+ * up to timeout_ms) and receive a duplicate of the served descriptor. */
+viper_status viper_debug_fd_listen(char *name_out, int32_t cap, int32_t *listen_fd);
+viper_status viper_debug_fd_serve(int32_t listen_fd, int32_t fd, int32_t n, int32_t timeout_ms);
+viper_status viper_debug_fd_fetch(const char *name, int32_t *fd_out, int64_t timeout_ms);
+
 /* Tear down (joins the update thread, frees library-owned memory). */
 viper_status viper_unregister(viper_model *m);
 

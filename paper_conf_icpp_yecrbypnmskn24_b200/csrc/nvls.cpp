@@ -143,6 +143,56 @@ size_t round_up(size_t x, size_t g) { return (x + g - 1) / g * g; }
 
 }  // namespace
 
+// ---- descriptor hand-off (no CUDA): an abstract Unix socket + SCM_RIGHTS.
+// fd_listen: a fresh name and a listening socket; fd_serve: hand `fd` to `n`
+// fetchers (bounded by timeout_ms per fetcher); fd_fetch: connect (retrying
+// until timeout_ns) and receive it.
+viper_status fd_listen(char *name, size_t cap, int *listen_fd) {
+    std::random_device rd;
+    snprintf(name, cap, "viper-nvls-%d-%08x", (int)getpid(), (unsigned)rd());
+    const int s = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
+    if (s < 0) return set_error(VIPER_E_UNSUPPORTED, "NVLS: socket() failed");
+    socklen_t len;
+    sockaddr_un a = sock_addr(name, &len);
+    if (bind(s, (sockaddr *)&a, len) != 0 || listen(s, 64) != 0) {
+        close(s);
+        return set_error(VIPER_E_UNSUPPORTED, "NVLS: cannot listen on @%s", name);
+    }
+    *listen_fd = s;
+    return VIPER_OK;
+}
+
+viper_status fd_serve(int listen_fd, int fd, int n, int timeout_ms) {
+    for (int k = 0; k < n; k++) {
+        pollfd p{listen_fd, POLLIN, 0};
+        if (poll(&p, 1, timeout_ms) != 1) return set_error(VIPER_E_PEER, "NVLS: fetcher %d did not connect", k);
+        const int c = accept(listen_fd, nullptr, nullptr);
+        if (c < 0) return set_error(VIPER_E_PEER, "NVLS: accept failed");
+        viper_status st = send_fd(c, fd);
+        close(c);
+        if (st) return st;
+    }
+    return VIPER_OK;
+}
+
+viper_status fd_fetch(const char *name, int *fd, int64_t timeout_ns) {
+    socklen_t len;
+    sockaddr_un a = sock_addr(name, &len);
+    const int64_t t0 = now_ns();
+    int s = -1;
+    for (;;) {
+        s = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
+        if (s >= 0 && connect(s, (sockaddr *)&a, len) == 0) break;
+        if (s >= 0) close(s);
+        s = -1;
+        if (now_ns() - t0 > timeout_ns) return set_error(VIPER_E_PEER, "NVLS: cannot reach @%s", name);
+        usleep(1000);
+    }
+    const viper_status st = recv_fd(s, fd);
+    close(s);
+    return st;
+}
+
 viper_status nvls_probe(int device) {
     std::call_once(g_drv_once, load_driver);
     if (!g_drv.ok) return set_error(VIPER_E_UNSUPPORTED, "NVLS: multicast driver entry points unavailable");
@@ -180,32 +230,14 @@ viper_status nvls_create(viper_model *m, int nranks, size_t bytes, char *sock_na
     int fd = -1;
     DRV_TRY(g_drv.exportFd(&fd, h, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0));
     m->nvls_fd = fd;
-    std::random_device rd;
-    snprintf(sock_name, cap, "viper-nvls-%d-%08x", (int)getpid(), (unsigned)rd());
-    const int s = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
-    if (s < 0) return set_error(VIPER_E_UNSUPPORTED, "NVLS: socket() failed");
-    socklen_t len;
-    sockaddr_un a = sock_addr(sock_name, &len);
-    if (bind(s, (sockaddr *)&a, len) != 0 || listen(s, 64) != 0) {
-        close(s);
-        return set_error(VIPER_E_UNSUPPORTED, "NVLS: cannot listen on @%s", sock_name);
-    }
-    m->nvls_listen = s;
-    return VIPER_OK;
+    return fd_listen(sock_name, cap, &m->nvls_listen);
 }
 
 // Producer: hand the fd to `nconsumers` connecting consumers, then add its own
 // device.  Bounded: a consumer that never connects fails the registration.
 viper_status nvls_serve(viper_model *m, int nconsumers) {
-    for (int k = 0; k < nconsumers; k++) {
-        pollfd p{m->nvls_listen, POLLIN, 0};
-        if (poll(&p, 1, 60000) != 1) return set_error(VIPER_E_PEER, "NVLS: consumer %d did not connect", k);
-        const int c = accept(m->nvls_listen, nullptr, nullptr);
-        if (c < 0) return set_error(VIPER_E_PEER, "NVLS: accept failed");
-        viper_status st = send_fd(c, m->nvls_fd);
-        close(c);
-        if (st) return st;
-    }
+    viper_status st = fd_serve(m->nvls_listen, m->nvls_fd, nconsumers, 60000);
+    if (st) return st;
     CUdevice d;
     DRV_TRY(g_drv.devGet(&d, m->device));
     DRV_TRY(g_drv.mcAddDevice((CUmemGenericAllocationHandle)m->nvls_mc, d));
@@ -217,21 +249,8 @@ viper_status nvls_join(viper_model *m, const char *sock_name, size_t bytes) {
     viper_status st = nvls_probe(m->device);
     if (st) return st;
     m->nvls_bytes = bytes;
-    int s = -1;
-    socklen_t len;
-    sockaddr_un a = sock_addr(sock_name, &len);
-    const int64_t t0 = now_ns();
-    for (;;) {
-        s = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
-        if (s >= 0 && connect(s, (sockaddr *)&a, len) == 0) break;
-        if (s >= 0) close(s);
-        s = -1;
-        if (now_ns() - t0 > 60ll * 1000000000ll) return set_error(VIPER_E_PEER, "NVLS: cannot reach @%s", sock_name);
-        usleep(1000);
-    }
     int fd = -1;
-    st = recv_fd(s, &fd);
-    close(s);
+    st = fd_fetch(sock_name, &fd, 60ll * 1000000000ll);
     if (st) return st;
     CUmemGenericAllocationHandle h;
     const CUresult r = g_drv.importFd(&h, (void *)(intptr_t)fd, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR);
@@ -303,3 +322,27 @@ void nvls_free(viper_model *m) {
 }
 
 }  // namespace vp
+
+// ---- test hooks (include/viper.h): the descriptor hand-off alone, no CUDA
+using namespace vp;
+extern "C" {
+viper_status viper_debug_fd_listen(char *name_out, int32_t cap, int32_t *listen_fd) {
+    if (!name_out || cap < 32 || !listen_fd) return set_error(VIPER_E_INVAL, "bad arguments");
+    int s = -1;
+    const viper_status st = fd_listen(name_out, (size_t)cap, &s);
+    *listen_fd = s;
+    return st;
+}
+viper_status viper_debug_fd_serve(int32_t listen_fd, int32_t fd, int32_t n, int32_t timeout_ms) {
+    const viper_status st = fd_serve(listen_fd, fd, n, timeout_ms);
+    close(listen_fd);
+    return st;
+}
+viper_status viper_debug_fd_fetch(const char *name, int32_t *fd_out, int64_t timeout_ms) {
+    if (!name || !fd_out) return set_error(VIPER_E_INVAL, "bad arguments");
+    int fd = -1;
+    const viper_status st = fd_fetch(name, &fd, timeout_ms * 1000000ll);
+    *fd_out = fd;
+    return st;
+}
+}

@@ -86,7 +86,7 @@ EXPORTS = ["viper_register_model", "viper_publish", "viper_subscribe", "viper_ac
            "viper_schedule", "viper_restore", "viper_strerror", "viper_last_error", "viper_version",
            "viper_debug_proto_create", "viper_debug_proto_open", "viper_debug_proto_close",
            "viper_debug_proto_publish", "viper_debug_proto_install", "viper_debug_proto_read",
-           "viper_debug_resolve_tier"]
+           "viper_debug_resolve_tier", "viper_debug_fd_listen", "viper_debug_fd_serve", "viper_debug_fd_fetch"]
 
 _lib = None
 _lock = threading.Lock()
@@ -138,6 +138,9 @@ def lib() -> C.CDLL:
                                                    C.POINTER(C.c_int32)]
             L.viper_restore.argtypes = [C.c_char_p, C.POINTER(viper_tensor), C.c_int32, C.c_int32, C.c_void_p,
                                         C.POINTER(C.c_uint64)]
+            L.viper_debug_fd_listen.argtypes = [C.c_char_p, C.c_int32, C.POINTER(C.c_int32)]
+            L.viper_debug_fd_serve.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.c_int32]
+            L.viper_debug_fd_fetch.argtypes = [C.c_char_p, C.POINTER(C.c_int32), C.c_int64]
             L.viper_strerror.argtypes = [C.c_int32]
             L.viper_strerror.restype = C.c_char_p
             L.viper_last_error.restype = C.c_char_p

@@ -241,3 +241,12 @@ def test_xproc_dram_install_does_not_hang_on_a_vanished_producer():
     producer unregisters: VIPER_E_PEER, v not installed, prompt unregister."""
     rc, out = run_torchrun(2, "tests/xproc_stall_worker.py", [], timeout=120)
     assert "STALL_CONSUMER" in out and "ok=True" in out, out[-4000:]
+
+
+def test_nvls_descriptor_handoff_gloo_cpu():
+    """The NVLS registration's fd hand-off (abstract Unix socket + SCM_RIGHTS),
+    CPU only: a served descriptor arrives in the other process and reads back
+    the same bytes; a missing fetcher / server fails with VIPER_E_PEER in
+    bounded time."""
+    rc, out = run_torchrun(2, "tests/fdpass_worker.py", [], timeout=120)
+    assert rc == 0 and "FDPASS rank0 ok=True" in out and "FDPASS rank1 ok=True" in out, out[-3000:]

@@ -20,6 +20,7 @@ ap.add_argument("--nofuse", action="store_true")
 ap.add_argument("--flags", type=int, default=0, help="extra VIPER_FLAG_* bits for the producer")
 ap.add_argument("--cflags", type=int, default=0, help="VIPER_FLAG_* bits for the consumer")
 ap.add_argument("--mode", type=int, default=0, help="0 SYNC, 1 ASYNC (the consumer's update thread installs)")
+ap.add_argument("--view-seals", action="store_true", help="seal the consumer's installed slot after every update")
 a = ap.parse_args()
 specs = synth.model_specs(a.config)
 seed = synth.SEEDS[a.config]
@@ -34,6 +35,12 @@ for v in range(1, a.steps + 1):
     p.publish(v)
     if a.mode == V.ASYNC:
         c.wait_installed(v)
+    if a.view_seals:
+        view = c.acquire_latest()
+        buf = torch.empty(16 * c.stats()["nchunks"], dtype=torch.uint8, device="cuda")
+        c.view_seals(view, buf)
+        torch.cuda.synchronize()
+        c.release(view)
 torch.cuda.synchronize()
 c.close()
 p.close()
