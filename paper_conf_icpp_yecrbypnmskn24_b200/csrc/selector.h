@@ -38,18 +38,22 @@ inline bool tier_reaches(const TierRec *all, int a, int b) {
 // `requested` unless it is VIPER_TIER_AUTO; then the GPU tier when every
 // consumer reaches every producer (ranks [producer_rank, producer_rank + M))
 // and -- with chain / scatter-allgather fan-out, where consumers also pull
-// from each other -- every other consumer; else the DRAM tier.  The
-// producers' own reach does not matter: nobody pulls from a consumer into a
-// producer.
+// from each other -- every other consumer; with push / NVLS fan-out, where
+// the producer writes into the consumers' memory, every producer must also
+// reach every consumer; else the DRAM tier.  Otherwise the producers' own
+// reach does not matter: nobody pulls from a consumer into a producer.
 inline int32_t resolve_tier(const TierRec *all, int world, int producer_rank, int M, int32_t fanout,
                             int32_t requested) {
     if (requested != VIPER_TIER_AUTO) return requested;
     auto producer = [&](int r) { return r >= producer_rank && r < producer_rank + M; };
     const bool peers = fanout == VIPER_FANOUT_CHAIN || fanout == VIPER_FANOUT_SCATTER_ALLGATHER;
+    const bool writes = fanout == VIPER_FANOUT_PUSH || fanout == VIPER_FANOUT_NVLS;
     for (int c = 0; c < world; c++) {
         if (producer(c)) continue;
-        for (int r = 0; r < world; r++)
+        for (int r = 0; r < world; r++) {
             if (r != c && (producer(r) || peers) && !tier_reaches(all, c, r)) return VIPER_TIER_DRAM;
+            if (writes && producer(r) && !tier_reaches(all, r, c)) return VIPER_TIER_DRAM;
+        }
     }
     return VIPER_TIER_GPU;
 }

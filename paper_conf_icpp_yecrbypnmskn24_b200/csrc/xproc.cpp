@@ -284,13 +284,24 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         st = set_error(VIPER_E_INVAL, "rank %d: role does not match bootstrap.producer_rank/nproducers", bs->rank);
     if (st == VIPER_OK && M > 1 && (m->cfg.tier != VIPER_TIER_GPU || m->cfg.fanout != VIPER_FANOUT_DIRECT))
         st = set_error(VIPER_E_UNSUPPORTED, "data-parallel producers: GPU tier, direct fan-out only");
-    const bool nvls = m->cfg.fanout == VIPER_FANOUT_NVLS;
-    const bool push = m->cfg.fanout == VIPER_FANOUT_PUSH;
+    // VIPER_TEST_NVLS_UNICAST=1 (tests, one consumer): NVLS registration without
+    // a multicast object -- the "multicast" address is the consumer's staging,
+    // mapped by CUDA IPC, and the producer's snapshot IS that buffer, as its
+    // share of the object would be.  On sm_100 multimem.st lowers to the same
+    // global store as a unicast one (the multicast is in the address
+    // mapping), so this runs pack_nvls_kernel and the consumer's NVLS install
+    // path bit for bit, everything but the switch's replication.
+    const char *emul_env = getenv("VIPER_TEST_NVLS_UNICAST");
+    const bool nvls_emul = m->cfg.fanout == VIPER_FANOUT_NVLS && emul_env && atoi(emul_env);
+    const bool nvls = m->cfg.fanout == VIPER_FANOUT_NVLS && !nvls_emul;
+    const bool push = m->cfg.fanout == VIPER_FANOUT_PUSH || nvls_emul;
     if (st == VIPER_OK && xproc_only_fanout(m->cfg.fanout) && m->cfg.tier != VIPER_TIER_GPU)
         st = set_error(VIPER_E_UNSUPPORTED, "fan-out %d needs the GPU tier (the Transfer Selector chose DRAM)",
                        m->cfg.fanout);
     if (st == VIPER_OK && push && bs->world - M > kMaxPush)
         st = set_error(VIPER_E_UNSUPPORTED, "push fan-out: at most %d consumers", kMaxPush);
+    if (st == VIPER_OK && nvls_emul && bs->world - M != 1)
+        st = set_error(VIPER_E_UNSUPPORTED, "VIPER_TEST_NVLS_UNICAST: exactly one consumer");
     if (st == VIPER_OK && nvls && !producer) st = nvls_probe(m->device);  // reported in allgather #1
     const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
     const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
@@ -420,6 +431,13 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             k++;
         }
         m->npush = k;
+        if (nvls_emul && st == VIPER_OK) {  // the snapshot and the "multicast" address: consumer 0's staging
+            for (int b = 0; b < 2; b++) {
+                m->d_snap[b] = m->nvls_mc_snap[b] = m->push_dst[b][0];
+                m->d_iseal[b] = m->nvls_mc_iseal[b] = m->push_iseal[b][0];
+            }
+            m->npush = 0;
+        }
     }
     if (st == VIPER_OK && producer && m->pidx > 0) {  // data-parallel producer j > 0: join the segment
         st = open_segment(m, pr.shm_path, pr.shm_bytes);

@@ -7,7 +7,7 @@ import ctypes as C
 
 MAGIC = 0x56495452
 GPU, DRAM, AUTO = 0, 1, 2
-DIRECT, CHAIN, SA = 0, 1, 2
+DIRECT, CHAIN, SA, NVLS, PUSH, CE = 0, 1, 2, 3, 4, 101
 
 
 class TierRec(C.Structure):
@@ -42,5 +42,9 @@ def reference(recs, devs, reach, producer_rank, M, fanout, requested, failed=())
             if c in failed or r in failed:
                 continue
             if devs[r] not in reach[c]:
+                return DRAM
+        # push / NVLS: the producers write into every consumer's memory
+        for p in prods:
+            if fanout in (PUSH, NVLS) and c not in failed and p not in failed and devs[c] not in reach[p]:
                 return DRAM
     return GPU

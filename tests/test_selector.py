@@ -85,7 +85,7 @@ def test_random_topologies_match_the_reference(seed):
             reach.append(sorted(s))
         failed = {r for r in range(world) if rng.random() < 0.05}
         requested = int(rng.choice([S.AUTO, S.AUTO, S.GPU, S.DRAM]))
-        fanout = int(rng.choice([S.DIRECT, S.CHAIN, S.SA]))
+        fanout = int(rng.choice([S.DIRECT, S.CHAIN, S.SA, S.PUSH, S.NVLS, S.CE]))
         recs = [S.TierRec() if r in failed else S.record(requested, devs[r], reach[r]) for r in range(world)]
         want = S.reference(recs, devs, reach, prank, M, fanout, requested, failed)
         assert resolve(recs, prank, M, fanout, requested) == want, (world, M, prank, devs, reach, fanout)
@@ -108,3 +108,17 @@ def test_records_over_gloo_world2(blocked, expect):
     r = subprocess.run(cmd, cwd=ROOT, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, timeout=120, text=True)
     assert r.returncode == 0, r.stdout[-3000:]
     assert r.stdout.count(f"SELECTOR {expect}") == 2, r.stdout[-3000:]
+
+
+def test_push_needs_the_producer_to_reach_every_consumer():
+    """Push / NVLS: the producer writes into the consumers' memory, so its GPU
+    must reach theirs; for pulls (direct, copy engine) only the consumers'
+    reach matters."""
+    # rank 0 = producer reaches only itself; consumers reach everything
+    recs = [S.record(S.AUTO, 0, [0]), S.record(S.AUTO, 1, [1, 0, 2]), S.record(S.AUTO, 2, [2, 0, 1])]
+    assert resolve(recs, fanout=S.DIRECT) == S.GPU
+    assert resolve(recs, fanout=S.CE) == S.GPU
+    assert resolve(recs, fanout=S.PUSH) == S.DRAM
+    assert resolve(recs, fanout=S.NVLS) == S.DRAM
+    full = [S.record(S.AUTO, i, [i] + [j for j in range(3) if j != i]) for i in range(3)]
+    assert resolve(full, fanout=S.PUSH) == S.GPU and resolve(full, fanout=S.NVLS) == S.GPU

@@ -250,3 +250,19 @@ def test_nvls_descriptor_handoff_gloo_cpu():
     bounded time."""
     rc, out = run_torchrun(2, "tests/fdpass_worker.py", [], timeout=120)
     assert rc == 0 and "FDPASS rank0 ok=True" in out and "FDPASS rank1 ok=True" in out, out[-3000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode,early,config", [(0, "0", "resnet50"), (1, "0", "small"), (0, "1", "resnet50"),
+                                              (1, "1", "ptychonn")])
+def test_xproc_nvls_kernel_path_unicast(mode, early, config):
+    """NVLS where the box has no multicast: VIPER_TEST_NVLS_UNICAST maps the
+    "multicast" address to the one consumer's staging (CUDA IPC) and makes it
+    the producer's snapshot, as its share of the object would be.  Runs
+    pack_nvls_kernel (multimem.st -- on sm_100 the same global store) and the
+    consumer's NVLS install path, with the early-notified item pipeline and
+    without; bit-exact slots and installed-slot seals == the oracle's."""
+    rc, out = run_torchrun(2, "tests/xproc_worker.py",
+                           ["--config", config, "--mode", str(mode), "--fanout", "3", "--versions", "5"],
+                           env={"VIPER_TEST_NVLS_UNICAST": "1", "VIPER_EARLY_NOTIFY": early})
+    assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
