@@ -293,6 +293,9 @@ typedef struct {
     uint64_t flushed, flush_skipped, flush_last;  /* producer with flush_dir        */
     int32_t tier;              /* tier in use (VIPER_TIER_AUTO resolved)               */
     int32_t fanout;            /* fan-out in use                                       */
+    double t_pickup_us;        /* consumer: producer's viper_publish entry -> this update
+                                  thread picked the version up (host CLOCK_MONOTONIC, shared by
+                                  every process on the node)                           */
 } viper_stats;
 viper_status viper_get_stats(viper_model *m, viper_stats *out);
 

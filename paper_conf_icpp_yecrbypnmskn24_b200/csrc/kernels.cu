@@ -291,6 +291,10 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
 // pack: stream every item tensor -> packed, write its item seal.  No atomics,
 // no fences: the consumer's kernel is ordered after this one by the stream /
 // event, which makes every store visible.
+#ifndef VP_PACK_UNROLL_SMALL
+#define VP_PACK_UNROLL_SMALL 8  // pack_seal's vectors per lane for snapshots <= 1 GiB (A/B: tune/ variants)
+#endif
+template <int U>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_kernel(const PackArgs a) {
     // let a programmatically-dependent install grid start now: it consumes
     // items as their ready flags flip (item-granular pack -> install pipeline)
@@ -305,8 +309,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_k
     for (; w < a.nitems; w += nwarps) {
         const Item it = nxt;  // descriptor prefetched one item ahead: its load overlaps this item's stream
         if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
-        const uint64_t part = warp_sum(copy_item<false>((const uint8_t *)it.ptr, a.packed + it.packed_off,
-                                                        it.nbytes, it.packed_off, lane, false));
+        const uint64_t part = warp_sum(copy_item<false, U>((const uint8_t *)it.ptr, a.packed + it.packed_off,
+                                                           it.nbytes, it.packed_off, lane, false));
         __syncwarp();  // every lane's stores are ordered before lane 0's release
         if (lane == 0) {
             ISeal *is = a.iseal + it.gidx;
@@ -462,6 +466,11 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_nvls_k
             mc_st_release_sys_u64(&a.mc_iseal[it.gidx].version, a.version);
         }
     }
+}
+
+// the pack instantiation for a snapshot of `bytes`
+static const void *pack_fn(uint64_t bytes) {
+    return bytes > (1ull << 30) ? (const void *)pack_seal_kernel<8> : (const void *)pack_seal_kernel<VP_PACK_UNROLL_SMALL>;
 }
 
 // chunk seals {version, sum of item checksums} -- one warp per chunk, off the
@@ -1454,8 +1463,8 @@ Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
     if (a.nitems == 0) return cudaSuccess;
-    pack_seal_kernel<<<g.grid, g.block, 0, st>>>(a);
-    return cudaGetLastError();
+    void *args[] = {(void *)&a};
+    return cudaLaunchKernel(pack_fn(a.s_packed), dim3(g.grid), dim3(g.block), args, 0, st);
 }
 
 cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
@@ -1501,7 +1510,7 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
         l.block = kTmaWarps * 32;
         l.smem = kTmaSmem;
     } else {
-        l.func = (const void *)pack_seal_kernel;
+        l.func = pack_fn(a.s_packed);
         l.grid = g.grid;
         l.block = g.block;
     }
@@ -1573,7 +1582,7 @@ cudaError_t preload_kernels() {
     const int dev = launch_device();
     const uint64_t bit = 1ull << (dev >= 0 && dev < kMaxDevices ? dev : 0);
     if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
-    const void *fns[] = {(const void *)pack_seal_kernel,         (const void *)seal_reduce_kernel,
+    const void *fns[] = {pack_fn(0), pack_fn(~0ull),              (const void *)seal_reduce_kernel,
                          (const void *)install_verify_kernel,    install_direct_fn(0, false),
                          install_direct_fn(~0ull, false),        install_direct_fn(0, true),
                          install_direct_fn(~0ull, true),

@@ -533,10 +533,19 @@ static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
     static const bool dbg_wait = getenv("VIPER_DEBUG") != nullptr;
     if (dbg_wait) fprintf(stderr, "[viper] waiting for the install of v%llu (slot %d)\n", (unsigned long long)v, b);
     for (uint32_t spins = 0;; spins++) {
-        const cudaError_t e = cudaStreamQuery(c->ustream);
-        if (e == cudaSuccess) return VIPER_OK;
-        if (e != cudaErrorNotReady) return set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
+        // the install kernel's last block reports in the mapped status word
+        // before the grid retires: the cheap, early signal (the stream query
+        // below covers errors and launches that never report)
+        if (c->rec->status.load() != 1) {
+            const cudaError_t e = cudaStreamSynchronize(c->ustream);
+            return e == cudaSuccess ? VIPER_OK : set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
+        }
         const int64_t dt = now_ns() - t0;
+        if ((spins & 63) == 63) {
+            const cudaError_t e = cudaStreamQuery(c->ustream);
+            if (e == cudaSuccess) return VIPER_OK;
+            if (e != cudaErrorNotReady) return set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
+        }
         if ((spins & 255) == 255) {
             viper_status why = VIPER_OK;
             if (c->stop.load()) why = set_error(VIPER_E_STATE, "install of v%llu abandoned: unregistering",
@@ -570,6 +579,11 @@ static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
     }
 }
 
+// How long an idle update thread spins on the control block before it sleeps
+// on the futex (VIPER_SPIN_US overrides): a futex wake-up costs tens of us of
+// scheduling latency, a spin costs a host core while it lasts.
+static const int64_t kIdleSpinNs = getenv("VIPER_SPIN_US") ? atoll(getenv("VIPER_SPIN_US")) * 1000 : 50000;
+
 void update_loop(viper_model *c) {
     cudaSetDevice(c->device);
     Ctrl *ctrl = c->ctrl;
@@ -592,11 +606,15 @@ void update_loop(viper_model *c) {
             }
         }
         if (!work) {
-            // short spin (notification latency), then sleep on the futex
+            // short spin (notification latency), then sleep on the futex.  The
+            // spin also watches the published word itself: an early-notified
+            // version is named by a stream memop on the producer's GPU, which
+            // may land after the host wake-up that roused this thread.
             const int64_t t0 = now_ns();
+            const uint64_t ps0 = ctrl->pub_state.load();
             bool got = false;
-            while (now_ns() - t0 < 50000) {
-                if (ctrl->pub_seq.load() != seq || c->stop.load()) {
+            while (now_ns() - t0 < kIdleSpinNs) {
+                if (ctrl->pub_seq.load() != seq || ctrl->pub_state.load() != ps0 || c->stop.load()) {
                     got = true;
                     break;
                 }
@@ -643,6 +661,8 @@ void update_loop(viper_model *c) {
         {
             std::lock_guard<std::mutex> sl(c->stats_mu);
             c->stats.t_notify_us = tp ? (t0 - tp) / 1e3 : 0.0;
+            const int64_t te = ctrl->pub_entry_ns.load(std::memory_order_relaxed);
+            c->stats.t_pickup_us = te ? (t0 - te) / 1e3 : 0.0;
         }
         lk.unlock();
         fire_callback(c, v, st);
@@ -721,6 +741,7 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         return set_error(VIPER_E_VERSION, "publish(%llu) after %llu: versions strictly increase from 1",
                          (unsigned long long)v, (unsigned long long)p->last_version);
     Ctrl *ctrl = p->ctrl;
+    ctrl->pub_entry_ns.store(t0, std::memory_order_relaxed);
     if (p->xproc && p->last_version) {
         // ASYNC cross-process: the previous version's notification (a host
         // function after its pack) must have named it before slot reuse
@@ -823,7 +844,9 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
         a.packed = p->d_snap[b];
         a.iseal = p->d_iseal[b];
         a.version = v;
-        a.sys_release = p->early_notify ? 1u : 0u;
+        static const bool force_sys = getenv("VIPER_TEST_SYS_RELEASE") && atoi(getenv("VIPER_TEST_SYS_RELEASE"));
+        a.sys_release = (p->early_notify || force_sys) ? 1u : 0u;  // (force: A/B of the seal release cost)
+        a.s_packed = p->man.s_packed;
         a.l2_once = fits_l2(p->device, p->man.s_packed) ? 1u : 0u;
         if (timing) CUDA_TRY(cudaEventRecord(p->ev_t[0], st));
         // a PDL-chained install must follow a plain stream launch; every

@@ -73,6 +73,7 @@ struct alignas(64) Ctrl {
     std::atomic<int32_t> nprod;
     std::atomic<int32_t> early_notify;   // producer names v before its pack completed
     std::atomic<int32_t> prod_pid;       // cross-process producer (liveness), 0 = in-process
+    std::atomic<int64_t> pub_entry_ns;   // CLOCK_MONOTONIC at the entry of the last viper_publish
 };
 
 // Pointer-free work item (the device lists add each endpoint's tensor address).

@@ -53,6 +53,7 @@ struct PackArgs {
                                 // on other GPUs pipeline behind this pack)
     uint32_t l2_once;           // TMA variant: load the tensors with an L2 evict-first hint
                                 // (set when the snapshot fits in L2, so it stays there)
+    uint64_t s_packed;          // packed size (selects the kernel instantiation)
 };
 
 // Push delivery (VIPER_FANOUT_PUSH): the pack also stores every item into

@@ -634,6 +634,14 @@ viper_status xproc_notify_early(viper_model *p, uint64_t v, int b, cudaStream_t 
         delete w;
         return set_error(VIPER_E_CUDA, "cudaLaunchHostFunc: %s", cudaGetErrorString(e));
     }
+    // ... and wake them from this thread now: when the stream is idle, the
+    // memop lands within microseconds, while a host function runs on the CUDA
+    // callback thread tens to hundreds of microseconds later
+    // (profiles/r02/notify_path.json).  A thread woken before the word lands
+    // spins on the word itself (update_loop); the host function above still
+    // wakes it if the stream reaches the pack only later.
+    p->ctrl->pub_seq.fetch_add(1);
+    futex_wake_all(&p->ctrl->pub_seq);
     return VIPER_OK;
 }
 

@@ -59,7 +59,7 @@ class viper_stats(C.Structure):
                 ("writer_wait_us", C.c_double), ("t_pack_dev_us", C.c_double),
                 ("t_install_dev_us", C.c_double), ("t_fused_dev_us", C.c_double), ("last_status", C.c_int32), ("nconsumers", C.c_int32),
                 ("flushed", C.c_uint64), ("flush_skipped", C.c_uint64), ("flush_last", C.c_uint64),
-                ("tier", C.c_int32), ("fanout", C.c_int32)]
+                ("tier", C.c_int32), ("fanout", C.c_int32), ("t_pickup_us", C.c_double)]
 
 
 class viper_sched_in(C.Structure):
