@@ -292,33 +292,21 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
 // no fences: the consumer's kernel is ordered after this one by the stream /
 // event, which makes every store visible.
 #ifndef VP_PACK_UNROLL_SMALL
-#define VP_PACK_UNROLL_SMALL 8  // pack_seal's vectors per lane for snapshots <= 1 GiB (A/B: tune/ variants)
+#define VP_PACK_UNROLL_SMALL 16  // pack_seal's vectors per lane for snapshots <= 1 GiB (profiles/r02/pack_ab.log)
 #endif
-template <int U>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_kernel(const PackArgs a) {
-    // let a programmatically-dependent install grid start now: it consumes
-    // items as their ready flags flip (item-granular pack -> install pipeline)
-    asm volatile("griddepcontrol.launch_dependents;");
-    const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
-    // Static strided items: measured faster than the work counter here
-    // (Llama-3 8B 5.05 vs 6.0 ms, profiles/r01/ktime_dynamic_ab.log).
-    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
-    Item nxt{};
-    if (w < a.nitems) nxt = a.items[w];
-    for (; w < a.nitems; w += nwarps) {
-        const Item it = nxt;  // descriptor prefetched one item ahead: its load overlaps this item's stream
-        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
-        const uint64_t part = warp_sum(copy_item<false, U>((const uint8_t *)it.ptr, a.packed + it.packed_off,
-                                                           it.nbytes, it.packed_off, lane, false));
-        __syncwarp();  // every lane's stores are ordered before lane 0's release
-        if (lane == 0) {
-            ISeal *is = a.iseal + it.gidx;
-            is->mixed = part + a.version * kVerMix;
-            if (a.sys_release) st_release_sys(&is->version, a.version);  // readers on other GPUs
-            else st_release(&is->version, a.version);  // item ready (pipelined install)
-        }
-    }
+
+// Item seals are released in batches of kRelBatch items per warp (pack_seal_kernel below).
+#ifndef VP_PACK_REL_BATCH
+#define VP_PACK_REL_BATCH 4
+#endif
+constexpr int kRelBatch = VP_PACK_REL_BATCH;
+
+__device__ __forceinline__ void st_relaxed_sys(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ void st_relaxed_gpu(uint64_t *p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 // ---------------------------------------------------------------------------
@@ -371,24 +359,43 @@ __device__ __forceinline__ uint64_t copy_item_push(const uint8_t *__restrict__ s
     return acc;
 }
 
+// Seals released in batches of kRelBatch items per warp, as in pack_seal
+// (one system-scope fence per batch instead of one per item and consumer).
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_push_kernel(const PushArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
-    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.p.nitems; w += nwarps) {
-        const Item it = a.p.items[w];
+    uint32_t pend_idx[kRelBatch];
+    int npend = 0;
+    auto release = [&]() {
+        if (lane == 0 && npend) {
+            asm volatile("fence.acq_rel.sys;" ::: "memory");  // the batch's data + cks words, everywhere
+#pragma unroll
+            for (int j = 0; j < kRelBatch; j++)
+                if (j < npend) {
+                    st_relaxed_sys(&a.p.iseal[pend_idx[j]].version, a.p.version);
+                    for (uint32_t k = 0; k < a.ndst; k++) st_relaxed_sys(&a.dst_iseal[k][pend_idx[j]].version, a.p.version);
+                }
+        }
+        npend = 0;
+    };
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    Item nxt{};
+    if (w < a.p.nitems) nxt = a.p.items[w];
+    for (; w < a.p.nitems; w += nwarps) {
+        const Item it = nxt;
+        if (w + nwarps < a.p.nitems) nxt = a.p.items[w + nwarps];
         const uint64_t part = warp_sum(copy_item_push((const uint8_t *)it.ptr, a.p.packed + it.packed_off, a,
                                                       it.packed_off, it.nbytes, lane));
-        __syncwarp();  // every lane's stores are ordered before lane 0's releases
+        __syncwarp();  // every lane's stores are ordered before lane 0's fence
         if (lane == 0) {
             const uint64_t mixed = part + a.p.version * kVerMix;
             a.p.iseal[it.gidx].mixed = mixed;
-            st_release(&a.p.iseal[it.gidx].version, a.p.version);
-            for (uint32_t k = 0; k < a.ndst; k++) {  // the consumers' copies of the seal, after the data
-                a.dst_iseal[k][it.gidx].mixed = mixed;
-                st_release_sys(&a.dst_iseal[k][it.gidx].version, a.p.version);
-            }
+            for (uint32_t k = 0; k < a.ndst; k++) a.dst_iseal[k][it.gidx].mixed = mixed;  // the consumers' copies
         }
+        pend_idx[npend++] = it.gidx;
+        if (npend == kRelBatch) release();
     }
+    release();
 }
 
 // ---------------------------------------------------------------------------
@@ -410,15 +417,30 @@ __device__ __forceinline__ void mc_st_u64(void *p, uint64_t v) {
     asm volatile("multimem.st.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
-__device__ __forceinline__ void mc_st_release_sys_u64(void *p, uint64_t v) {
-    asm volatile("multimem.st.release.sys.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+__device__ __forceinline__ void mc_st_relaxed_sys_u64(void *p, uint64_t v) {
+    asm volatile("multimem.st.relaxed.sys.global.b64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_nvls_kernel(const NvlsArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
-    for (uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5); w < a.nitems; w += nwarps) {
-        const Item it = a.items[w];
+    uint32_t pend_idx[kRelBatch];  // seals released in batches (pack_seal)
+    int npend = 0;
+    auto release = [&]() {
+        if (lane == 0 && npend) {
+            asm volatile("fence.acq_rel.sys;" ::: "memory");
+#pragma unroll
+            for (int j = 0; j < kRelBatch; j++)
+                if (j < npend) mc_st_relaxed_sys_u64(&a.mc_iseal[pend_idx[j]].version, a.version);
+        }
+        npend = 0;
+    };
+    uint32_t w0 = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    Item nxt{};
+    if (w0 < a.nitems) nxt = a.items[w0];
+    for (uint32_t w = w0; w < a.nitems; w += nwarps) {
+        const Item it = nxt;
+        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
         const uint8_t *src = (const uint8_t *)it.ptr;
         uint8_t *dst = a.mc_packed + it.packed_off;
         const uint32_t n = it.nbytes;
@@ -460,17 +482,71 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_nvls_k
         }
         const uint64_t part = warp_sum(acc);
         __syncwarp();
-        if (lane == 0) {
-            mc_st_u64(&a.mc_iseal[it.gidx].mixed, part + a.version * kVerMix);
-            asm volatile("fence.acq_rel.sys;" ::: "memory");
-            mc_st_release_sys_u64(&a.mc_iseal[it.gidx].version, a.version);
-        }
+        if (lane == 0) mc_st_u64(&a.mc_iseal[it.gidx].mixed, part + a.version * kVerMix);
+        pend_idx[npend++] = it.gidx;
+        if (npend == kRelBatch) release();
     }
+    release();
 }
 
-// the pack instantiation for a snapshot of `bytes`
-static const void *pack_fn(uint64_t bytes) {
-    return bytes > (1ull << 30) ? (const void *)pack_seal_kernel<8> : (const void *)pack_seal_kernel<VP_PACK_UNROLL_SMALL>;
+// pack: stream every item tensor -> packed and seal it.  The seals are what a
+// pipelined install waits on: a PDL-chained install on this GPU (gpu scope) or,
+// under early notification, consumers on OTHER GPUs (kSys: system scope).  A
+// release costs lane 0 a fence (MEMBAR.GPU / MEMBAR.SYS) that stalls the warp,
+// and the system-scope one is expensive: one per 8-KiB item made the pack 1.4-
+// 1.8x slower (profiles/r02/pack_release_ab.log).  So the seals are released
+// in batches of kRelBatch items per warp: lane 0 writes the batch's cks words,
+// issues ONE fence, then the versions as relaxed stores (the fence + relaxed
+// store pair is a release: a consumer that acquires a version sees its item's
+// data and cks).  Items stay the pipeline's unit; a seal just becomes visible
+// up to kRelBatch - 1 items later.  The __syncwarp after each item orders
+// every lane's stores before lane 0's fence.  Static strided items (measured
+// faster than the work counter here: Llama-3 8B 5.05 vs 6.0 ms,
+// profiles/r01/ktime_dynamic_ab.log), descriptors prefetched one item ahead.
+template <int U, bool kSys>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) pack_seal_kernel(const PackArgs a) {
+    // let a programmatically-dependent install grid start now: it consumes
+    // items as their ready flags flip (item-granular pack -> install pipeline)
+    asm volatile("griddepcontrol.launch_dependents;");
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
+    uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    uint32_t pend_idx[kRelBatch];
+    int npend = 0;
+    auto release = [&]() {  // lane 0: one fence for the batch, then its versions
+        if (lane == 0 && npend) {
+            if (kSys) asm volatile("fence.acq_rel.sys;" ::: "memory");
+            else asm volatile("fence.acq_rel.gpu;" ::: "memory");
+#pragma unroll
+            for (int k = 0; k < kRelBatch; k++)
+                if (k < npend) {
+                    if (kSys) st_relaxed_sys(&a.iseal[pend_idx[k]].version, a.version);
+                    else st_relaxed_gpu(&a.iseal[pend_idx[k]].version, a.version);
+                }
+        }
+        npend = 0;
+    };
+    Item nxt{};
+    if (w < a.nitems) nxt = a.items[w];
+    for (; w < a.nitems; w += nwarps) {
+        const Item it = nxt;  // descriptor prefetched one item ahead: its load overlaps this item's stream
+        if (w + nwarps < a.nitems) nxt = a.items[w + nwarps];
+        const uint64_t part = warp_sum(copy_item<false, U>((const uint8_t *)it.ptr, a.packed + it.packed_off,
+                                                           it.nbytes, it.packed_off, lane, false));
+        __syncwarp();  // every lane's stores are ordered before lane 0's fence
+        if (lane == 0) a.iseal[it.gidx].mixed = part + a.version * kVerMix;  // before the fence, too
+        pend_idx[npend++] = it.gidx;
+        if (npend == kRelBatch) release();
+    }
+    release();
+}
+
+// the pack instantiation for a snapshot of `bytes` (sys: seals released at system scope)
+static const void *pack_fn(uint64_t bytes, bool sys = false) {
+    const bool big = bytes > (1ull << 30);
+    if (sys)
+        return big ? (const void *)pack_seal_kernel<8, true> : (const void *)pack_seal_kernel<VP_PACK_UNROLL_SMALL, true>;
+    return big ? (const void *)pack_seal_kernel<8, false> : (const void *)pack_seal_kernel<VP_PACK_UNROLL_SMALL, false>;
 }
 
 // chunk seals {version, sum of item checksums} -- one warp per chunk, off the
@@ -606,6 +682,27 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
     bool bad = false;
     uint32_t w = blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     WorkQueue q(a.ctr, 0, nwarps, a.nitems);  // reset by the last block (install_finish)
+    // Items staged for the peers (scatter-allgather owner / chain link) have
+    // their seals released in batches of kRelBatch (one system-scope fence per
+    // batch, as in pack_seal), but never held across a wait: a warp that is
+    // about to wait for a seal first releases what it holds, so two consumers
+    // can never wait on each other's pending seals.
+    uint32_t rp_idx[kRelBatch];
+    int rp_n = 0;
+    auto release_staged = [&]() {
+        if (lane == 0 && rp_n) {
+            asm volatile("fence.acq_rel.sys;" ::: "memory");
+#pragma unroll
+            for (int j = 0; j < kRelBatch; j++)
+                if (j < rp_n) st_relaxed_sys(&a.sa_iseal_out[rp_idx[j]].version, a.version);
+        }
+        rp_n = 0;
+    };
+    auto ready = [&](const ISeal *x) {  // warp-uniform: lane 0's first look at a seal
+        int r = 0;
+        if (lane == 0) r = ld_acquire_sys(&x->version) == a.version;
+        return __shfl_sync(0xffffffffu, r, 0) != 0;
+    };
     if (w < a.nitems) q.claim(lane);
     while (w < a.nitems) {
         const Item it = a.items[w];
@@ -640,6 +737,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             }
         }
         if (peer >= 0) {
+            if (!ready(a.sa_isrc[peer] + w)) release_staged();
             int ok = 0;
             if (lane == 0) {
                 const ISeal *ps = a.sa_isrc[peer] + w;
@@ -665,6 +763,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             }
         }
         // (system scope: the producer may be another GPU pipelining its pack)
+        if (rp_n && !ready(is)) release_staged();
         uint64_t expect = 0;
         if (lane == 0) {
             uint32_t backoff = 32;
@@ -709,19 +808,24 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                 from_peer = false;
                 continue;
             }
+            __syncwarp();  // every lane's staging stores before lane 0's (batched) release
             if (lane == 0) {
-                if (republish) {  // peers may now pull item w from this consumer's staging
+                if (republish) {  // peers may pull item w from this consumer's staging once released
                     a.sa_iseal_out[w].mixed = expect;
-                    st_release_sys(&a.sa_iseal_out[w].version, a.version);
                     if (staged + a.version * kVerMix != expect) bad = true;
                 }
                 if (part + a.version * kVerMix != expect) bad = true;
+            }
+            if (republish) {
+                rp_idx[rp_n++] = w;
+                if (rp_n == kRelBatch) release_staged();
             }
             break;
         }
         w = q.next(w, lane);
         if (w < a.nitems) q.claim(lane);
     }
+    release_staged();
     install_finish(a, bad);
 }
 
@@ -1464,7 +1568,7 @@ Geometry pick_geometry(uint32_t nitems, int device, int max_sms) {
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
     if (a.nitems == 0) return cudaSuccess;
     void *args[] = {(void *)&a};
-    return cudaLaunchKernel(pack_fn(a.s_packed), dim3(g.grid), dim3(g.block), args, 0, st);
+    return cudaLaunchKernel(pack_fn(a.s_packed, a.sys_release), dim3(g.grid), dim3(g.block), args, 0, st);
 }
 
 cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
@@ -1510,7 +1614,7 @@ LaunchSpec pack_launch(const PackArgs &a, const Geometry &g, bool tma, int devic
         l.block = kTmaWarps * 32;
         l.smem = kTmaSmem;
     } else {
-        l.func = pack_fn(a.s_packed);
+        l.func = pack_fn(a.s_packed, a.sys_release);
         l.grid = g.grid;
         l.block = g.block;
     }
@@ -1582,7 +1686,8 @@ cudaError_t preload_kernels() {
     const int dev = launch_device();
     const uint64_t bit = 1ull << (dev >= 0 && dev < kMaxDevices ? dev : 0);
     if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
-    const void *fns[] = {pack_fn(0), pack_fn(~0ull),              (const void *)seal_reduce_kernel,
+    const void *fns[] = {pack_fn(0), pack_fn(~0ull), pack_fn(0, true), pack_fn(~0ull, true),
+                         (const void *)seal_reduce_kernel,
                          (const void *)install_verify_kernel,    install_direct_fn(0, false),
                          install_direct_fn(~0ull, false),        install_direct_fn(0, true),
                          install_direct_fn(~0ull, true),
