@@ -1222,19 +1222,13 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
     bool bad = false;
     for (uint32_t w = w0; w < a.nitems; w += nwarps) {
         const Item it = a.items[w];
-        uint64_t expect = 0;
-        if (lane == 0) {  // not PDL-chained: the seal is already there; still never hang
-            const ISeal *is = a.iseal + w;
-            uint64_t waited = 0;
-            while (ld_acquire_sys(&is->version) != a.version) {
-                __nanosleep(256);
-                if ((waited += 256) > kItemWaitNs || wait_aborted(a)) {
-                    report_err(a.flags, kErrTimeout);
-                    break;
-                }
-            }
-            expect = is->mixed;
-        }
+        // Only complete snapshots come here (not PDL-chained, not early-notified):
+        // the seal is already there, so it is loaded now and checked when the
+        // item is done instead of stalling lane 0 -- which issues the warp's
+        // bulk copies -- on a round trip per item (the acquire spin below is
+        // the never-hang fallback, not the expected path).
+        ISeal sl{};
+        if (lane == 0) sl = ld_seal(a.iseal + w);
         const uint32_t body = body_of(it);
         uint64_t acc = 0;
         for (uint32_t off = 0; off < body; off += kTmaStage) {
@@ -1271,7 +1265,10 @@ __global__ void __launch_bounds__(kTmaWarps * 32, 2) install_verify_tma_kernel(c
                                : copy_words_bytewise<true>(a.packed + it.packed_off, (uint8_t *)it.ptr, body,
                                                            it.nbytes, it.packed_off, lane, false);
         const uint64_t part = warp_sum(acc);
-        if (lane == 0 && part + a.version * kVerMix != expect) bad = true;
+        if (lane == 0) {
+            const uint64_t expect = sl.version == a.version ? sl.mixed : acquire_seal(a, w);
+            if (part + a.version * kVerMix != expect) bad = true;
+        }
     }
     if (lane == 0)  // slot stores complete, then ordered before the generic-proxy release below
         asm volatile("cp.async.bulk.wait_group 0;\n\tfence.proxy.async.global;" ::: "memory");
