@@ -738,10 +738,10 @@ def xproc_e2e(V, G, synth, name, rank, world, dev, group, fanout, flush_buf, ste
 
 # include/viper.h VIPER_FANOUT_*; "dram" (-1) = the pinned-DRAM tier (BASELINE configs[4]: DRAM-to-DRAM
 # staging vs direct GPU-to-GPU), direct fan-out
-FANOUTS = {"direct": 0, "chain": 1, "sa": 2, "nvls": 3, "push": 4, "ce": 101, "dram": -1}
+FANOUTS = {"direct": 0, "chain": 1, "sa": 2, "nvls": 3, "push": 4, "nccl": 100, "ce": 101, "dram": -1}
 FANOUT_NAMES = {0: "direct pull", 1: "pipelined chain", 2: "scatter-allgather", 3: "NVLS multicast",
-                4: "push (producer stores into peer staging)", 101: "copy engine (engine baseline)",
-                -1: "pinned-DRAM tier (D2H -> shared host staging -> H2D)"}
+                4: "push (producer stores into peer staging)", 100: "NCCL broadcast (engine baseline)",
+                101: "copy engine (engine baseline)", -1: "pinned-DRAM tier (D2H -> shared host staging -> H2D)"}
 NVLINK_GBS = 900.0  # NVLink 5 per direction per GPU (north_star / B200_PROFILING.md)
 
 
@@ -1109,11 +1109,11 @@ def xproc_arm(args):
     if args.fanout != "auto":
         order = [args.fanout]
     elif world == 2:
-        order = ["direct", "push", "ce", "nvls", "dram"]
+        order = ["direct", "push", "nvls", "ce", "nccl", "dram"]
     else:
-        order = ["nvls", "sa", "chain", "push", "direct", "ce", "dram"]
+        order = ["nvls", "sa", "chain", "push", "direct", "ce", "nccl", "dram"]
     if over and args.fanout == "auto":  # ranks time-slice one GPU: peer waits only serialise
-        order = ["direct", "push", "ce", "dram"]
+        order = ["direct", "push", "ce", "nccl", "dram"]
     results = {}
     with ClockSampler(dev) as clk:
         for f in order:
@@ -1126,8 +1126,9 @@ def xproc_arm(args):
     # headline: the first fan-out in preference order that ran and verified bit-exact (rank 0 decides)
     head = None
     if rank == 0:
-        head = next((f for f in order if f != "dram" and results[f].get("parity_ok")), None)
-        head = head or next((f for f in order if f != "dram" and "latency_ms" in results[f]), order[0])
+        engine = [f for f in order if f not in ("dram", "nccl", "ce")]  # the baselines never headline
+        head = next((f for f in engine if results[f].get("parity_ok")), None)
+        head = head or next((f for f in engine if "latency_ms" in results[f]), engine[0] if engine else order[0])
     head = gather_obj(head, gloo)[0]
     log(f"fan-outs timed, headline {head}; baselines")
     # baselines on the same bytes: NCCL broadcast (device time, max over ranks) and a torch copy-engine pull

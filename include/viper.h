@@ -129,16 +129,22 @@ enum { VIPER_FANOUT_DIRECT = 0,        /* every consumer pulls every chunk from 
                                           (producer egress N x S, at most 8 consumers);
                                           consumers install from local HBM, item by item
                                           as the producer releases the item seals */
-       VIPER_FANOUT_NCCL = 100,        /* baseline: reserved; bench.py times
-                                          torch.distributed.broadcast over NCCL instead.
-                                          Registration returns VIPER_E_UNSUPPORTED */
+       VIPER_FANOUT_NCCL = 100,        /* baseline as an engine transport: after
+                                          its pack the producer broadcasts the sealed snapshot
+                                          and its item seals with NCCL (libnccl.so.2,
+                                          dlopen'ed; VIPER_NCCL_LIB overrides); each consumer
+                                          receives them into its staging and installs +
+                                          verifies locally.  SYNC only (a broadcast is a
+                                          lock-step collective), one GPU per rank; otherwise
+                                          registration returns VIPER_E_UNSUPPORTED on every
+                                          rank */
        VIPER_FANOUT_CE = 101           /* baseline: each consumer's update
                                           thread copies the sealed snapshot with the copy
                                           engine (cudaMemcpyAsync peer -> local staging)
                                           once the pack completed, then installs locally */
 };
-/* NVLS, PUSH and CE are cross-process fan-outs (viper_bootstrap != NULL, GPU
- * tier, one producer); in process they return VIPER_E_UNSUPPORTED. */
+/* NVLS, PUSH, NCCL and CE are cross-process fan-outs (viper_bootstrap != NULL,
+ * GPU tier, one producer); in process they return VIPER_E_UNSUPPORTED. */
 /* Save mode (Fig. 3; s5.3 P:2143-2153). */
 enum { VIPER_SYNC = 0,   /* publish returns after every consumer installed v (or failed) */
        VIPER_ASYNC = 1 };/* publish returns once the snapshot is enqueued on cuda_stream;

@@ -17,7 +17,7 @@ CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libviper.so")
 VGEN_SRC = os.path.join(ROOT, "synth", "vgen.cu")
 VGEN_LIB = os.path.join(ROOT, "synth", "libvgen.so")
-SOURCES = ["kernels.cu", "runtime.cpp", "schedule.cpp", "xproc.cpp", "flush.cpp", "selftest.cpp", "nvls.cpp"]
+SOURCES = ["kernels.cu", "runtime.cpp", "schedule.cpp", "xproc.cpp", "flush.cpp", "selftest.cpp", "nvls.cpp", "nccl_fanout.cpp"]
 HEADERS = ["vp_internal.h", "runtime.h", "protocol.h", "selector.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -61,7 +61,7 @@ def build_viper(force: bool = False, verbose: bool = False, out: str = None, def
         if verbose and log.strip():
             print(log)
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread", "-lrt"]
+    cmd = [nvcc()] + ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread", "-lrt", "-ldl"]
     r = subprocess.run(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)
     if r.returncode != 0:
         raise RuntimeError("link failed:\n" + r.stdout.decode())

@@ -365,7 +365,7 @@ viper_status prepare_install(viper_model *c, const SnapSource &src, uint64_t v, 
     a = InstallArgs{};
     // DRAM tier / copy-engine baseline: the install reads this GPU's staging,
     // filled by the copies launch_prepared enqueues ahead of the kernel
-    const bool staged = c->cfg.tier == VIPER_TIER_DRAM || c->cfg.fanout == VIPER_FANOUT_CE;
+    const bool staged = copy_staged(c->cfg.tier, c->cfg.fanout);
     a.items = c->d_slot_items[target];
     a.nitems = (uint32_t)c->man.items.size();
     a.packed = staged ? c->d_stage : src.snap[b];
@@ -420,6 +420,11 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
         CUDA_TRY(cudaMemcpyAsync(c->d_stage, src.snap[b], c->man.s_packed, cudaMemcpyDefault, st));
         CUDA_TRY(cudaMemcpyAsync(c->d_stage_iseal, src.iseal[b], sizeof(ISeal) * c->man.items.size(),
                                  cudaMemcpyDefault, st));
+        pdl = false;
+    } else if (c->cfg.fanout == VIPER_FANOUT_NCCL) {
+        // NCCL baseline: receive the producer's broadcasts of v into the staging
+        viper_status s = nccl_broadcast_version(c, c->d_stage, c->d_stage_iseal, c->nccl_root, st);
+        if (s) return s;
         pdl = false;
     } else if (wait_ready && src.ev_ready[b]) {
         CUDA_TRY(cudaStreamWaitEvent(st, src.ev_ready[b], 0));
@@ -912,6 +917,12 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     }
     // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
+    if (p->cfg.fanout == VIPER_FANOUT_NCCL) {
+        // NCCL baseline: broadcast v to the consumers' staging, AFTER ev_packed:
+        // the notification that lets them join the collective waits on it
+        viper_status s = nccl_broadcast_version(p, p->d_snap[b], p->d_iseal[b], p->rank, st);
+        if (s) return s;
+    }
     CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
     if (p->xproc && !sync && !p->early_notify) {
         // remote consumers read slot b without events: name v once the pack is
@@ -1119,7 +1130,7 @@ viper_status alloc_consumer(viper_model *m, const viper_tensor *tensors) {
         if ((st = upload_items(m->man, m->slot_ptrs[s], &m->d_slot_items[s], 1, 0, nullptr))) return st;
     CUDA_TRY(cudaMalloc(&m->d_flags, 64));
     CUDA_TRY(cudaMemset(m->d_flags, 0, 64));
-    if (m->cfg.tier == VIPER_TIER_DRAM || m->cfg.fanout == VIPER_FANOUT_CE) {
+    if (copy_staged(m->cfg.tier, m->cfg.fanout)) {
         const uint64_t IS = al256(sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1));
         CUDA_TRY(cudaMalloc(&m->stage_alloc, al256(S) + IS));
         m->d_stage = (uint8_t *)m->stage_alloc;
@@ -1275,14 +1286,11 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
             return set_error(VIPER_E_INVAL, "bad tier");
         if (c.mode != VIPER_SYNC && c.mode != VIPER_ASYNC) return set_error(VIPER_E_INVAL, "bad mode");
         if (c.install_sms < 0) return set_error(VIPER_E_INVAL, "install_sms must be >= 0");
-        if (c.fanout == VIPER_FANOUT_NCCL)
-            return set_error(VIPER_E_UNSUPPORTED, "fanout NCCL is a bench.py baseline (torch.distributed.broadcast), "
-                                                  "not an engine transport");
         if (c.fanout != VIPER_FANOUT_DIRECT && c.fanout != VIPER_FANOUT_CHAIN &&
             c.fanout != VIPER_FANOUT_SCATTER_ALLGATHER && !xproc_only_fanout(c.fanout))
             return set_error(VIPER_E_UNSUPPORTED, "fanout %d not supported", c.fanout);
         if (xproc_only_fanout(c.fanout) && !(bs && bs->world > 1))
-            return set_error(VIPER_E_UNSUPPORTED, "fanout %d (NVLS / push / CE) needs the cross-process channel",
+            return set_error(VIPER_E_UNSUPPORTED, "fanout %d (NVLS / push / CE / NCCL) needs the cross-process channel",
                              c.fanout);
         int ndev = 0;
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0)

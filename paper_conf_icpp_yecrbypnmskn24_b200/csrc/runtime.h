@@ -32,7 +32,12 @@ constexpr uint64_t kCtrlMagic = 0x5649504552435431ull;  // "VIPERCT1"
 
 // Fan-outs that exist only across processes (one producer, GPU tier).
 inline bool xproc_only_fanout(int32_t f) {
-    return f == VIPER_FANOUT_NVLS || f == VIPER_FANOUT_PUSH || f == VIPER_FANOUT_CE;
+    return f == VIPER_FANOUT_NVLS || f == VIPER_FANOUT_PUSH || f == VIPER_FANOUT_CE || f == VIPER_FANOUT_NCCL;
+}
+// Consumers receive the snapshot into a device staging buffer by a copy ahead of
+// the install (DRAM tier: H2D; copy engine: peer copy; NCCL: broadcast).
+inline bool copy_staged(int32_t tier, int32_t f) {
+    return tier == VIPER_TIER_DRAM || f == VIPER_FANOUT_CE || f == VIPER_FANOUT_NCCL;
 }
 // Consumers install from a local staging buffer the producer writes into
 // (push: peer stores; NVLS: multicast stores).
@@ -223,6 +228,8 @@ struct viper_model {
     int nvls_fd = -1, nvls_listen = -1;
     bool nvls_have_mc = false, nvls_have_phys = false, nvls_bound = false, nvls_uc_mapped = false,
          nvls_mc_mapped = false;
+    void *nccl_comm = nullptr;                       // VIPER_FANOUT_NCCL: the communicator (ncclComm_t)
+    int32_t nccl_root = 0;                           // the producer's rank in it
     uint8_t *nvls_mc_snap[2] = {nullptr, nullptr};   // producer: multicast VA of snapshot slot b
     vp::ISeal *nvls_mc_iseal[2] = {nullptr, nullptr};
 
@@ -302,5 +309,11 @@ viper_status nvls_serve(viper_model *m, int nconsumers);                        
 viper_status nvls_join(viper_model *m, const char *sock_name, size_t bytes);                      // consumer
 viper_status nvls_bind(viper_model *m, bool map_mc);                                              // every rank
 void nvls_free(viper_model *m);
+
+// nccl_fanout.cpp (VIPER_FANOUT_NCCL, the NCCL-broadcast baseline as an engine transport)
+viper_status nccl_probe(void *unique_id_out);  // unique_id_out: 128 B (producer) or NULL
+viper_status nccl_init(viper_model *m, const void *unique_id, int world, int rank);
+viper_status nccl_broadcast_version(viper_model *m, void *snap, void *iseal, int root, cudaStream_t st);
+void nccl_free(viper_model *m);
 
 }  // namespace vp

@@ -49,6 +49,7 @@ struct PeerRec {
     char pci[32];                            // PCI bus id of the rank's GPU
     char nvls_sock[64];                      // producer, NVLS: abstract socket serving the multicast fd
     uint64_t nvls_bytes;                     // producer, NVLS: size of the multicast object
+    char nccl_id[128];                       // producer, NCCL fan-out: the ncclUniqueId
 };
 
 uint64_t fnv1a(const void *p, size_t n, uint64_t h = 0xcbf29ce484222325ull) {
@@ -303,6 +304,10 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
     if (st == VIPER_OK && nvls_emul && bs->world - M != 1)
         st = set_error(VIPER_E_UNSUPPORTED, "VIPER_TEST_NVLS_UNICAST: exactly one consumer");
     if (st == VIPER_OK && nvls && !producer) st = nvls_probe(m->device);  // reported in allgather #1
+    const bool nccl = m->cfg.fanout == VIPER_FANOUT_NCCL;
+    if (st == VIPER_OK && nccl && producer && m->cfg.mode != VIPER_SYNC)
+        st = set_error(VIPER_E_UNSUPPORTED, "NCCL fan-out: SYNC only (broadcasts are a lock-step collective)");
+    if (st == VIPER_OK && nccl) st = nccl_probe(producer ? (void *)me.nccl_id : nullptr);  // reported in #1
     const uint64_t S = (m->man.s_packed + 255) / 256 * 256;
     const uint64_t IS = (sizeof(ISeal) * std::max<size_t>(m->man.items.size(), 1) + 255) / 256 * 256;
     const size_t ctrl_bytes = page_up(sizeof(Ctrl));
@@ -373,11 +378,12 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
                 st = set_error(VIPER_E_INVAL, "rank %d uses another tier / fan-out", r);
         }
     }
-    if (st == VIPER_OK && nvls) {  // NVLS binds one buffer per GPU: ranks must not share a GPU
+    if (st == VIPER_OK && (nvls || nccl)) {  // NVLS / NCCL: one GPU per rank
         for (int r = 0; r < bs->world && st == VIPER_OK; r++)
             for (int q = r + 1; q < bs->world; q++)
                 if (strncmp(all[r].pci, all[q].pci, sizeof me.pci) == 0) {
-                    st = set_error(VIPER_E_UNSUPPORTED, "NVLS: ranks %d and %d share GPU %s", r, q, all[r].pci);
+                    st = set_error(VIPER_E_UNSUPPORTED, "%s: ranks %d and %d share GPU %s", nvls ? "NVLS" : "NCCL",
+                                   r, q, all[r].pci);
                     break;
                 }
     }
@@ -395,6 +401,10 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (ms[r].status != VIPER_OK)
                 st = set_error(ms[r].status == VIPER_E_UNSUPPORTED ? VIPER_E_UNSUPPORTED : VIPER_E_PEER,
                                "rank %d failed to register", r);
+    }
+    if (st == VIPER_OK && nccl) {  // every rank is known to be fine: the collective init cannot strand one
+        m->nccl_root = bs->producer_rank;
+        st = nccl_init(m, pr.nccl_id, bs->world, bs->rank);
     }
     if (st == VIPER_OK && nvls) {
         st = nvls_bind(m, producer);
@@ -451,7 +461,8 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
             if (all[r].role != VIPER_PRODUCER && strncmp(all[r].pci, me.pci, sizeof me.pci) == 0) other = false;
         const char *env = getenv("VIPER_EARLY_NOTIFY");
         m->early_notify = env ? atoi(env) != 0 : other;
-        if (m->cfg.fanout == VIPER_FANOUT_CE) m->early_notify = false;  // the copy engine needs a sealed snapshot
+        // the copy engine and NCCL move a sealed snapshot
+        if (m->cfg.fanout == VIPER_FANOUT_CE || m->cfg.fanout == VIPER_FANOUT_NCCL) m->early_notify = false;
         if (m->pidx == 0) m->ctrl->early_notify.store(m->early_notify ? 1 : 0);
     }
     if (st == VIPER_OK && !producer) {
@@ -654,6 +665,7 @@ void xproc_free(viper_model *m) {
     for (auto &p : m->push_peer_base)
         if (p) cudaIpcCloseMemHandle(p), p = nullptr;
     nvls_free(m);
+    nccl_free(m);
     cudaFree(m->d_mp_tab);
     m->d_mp_tab = nullptr;
     cudaFree(m->d_sa_tab);

@@ -222,6 +222,21 @@ def test_xproc_push_fault():
 
 
 @pytest.mark.gpu
+@pytest.mark.parametrize("nproc,mode", [(2, 0), (3, 0), (2, 1)])
+def test_xproc_nccl_bit_exact_or_unsupported_everywhere(nproc, mode):
+    """VIPER_FANOUT_NCCL (the NCCL-broadcast baseline inside the engine):
+    bit-exact with one GPU per rank and SYNC; ranks sharing a GPU (NCCL refuses
+    that) or an ASYNC producer give VIPER_E_UNSUPPORTED on every rank."""
+    rc, out = run_torchrun(nproc, "tests/xproc_worker.py",
+                           ["--config", "resnet50", "--fanout", "100", "--mode", str(mode), "--versions", "4",
+                            "--allow-unsupported"])
+    assert rc == 0, out[-4000:]
+    assert "XPROC_RESULT errors=0" in out or "XPROC_UNSUPPORTED everywhere=True" in out, out[-4000:]
+    if mode == 1:
+        assert "XPROC_UNSUPPORTED everywhere=True" in out, out[-4000:]
+
+
+@pytest.mark.gpu
 @pytest.mark.parametrize("nproc", [2, 3])
 def test_xproc_nvls_bit_exact_or_unsupported_everywhere(nproc):
     """VIPER_FANOUT_NVLS: bit-exact where the box exposes multicast (one GPU per
