@@ -219,20 +219,20 @@ __device__ __forceinline__ uint64_t copy_item(const uint8_t *__restrict__ src, u
 // (same lane, same addresses -> ordered; an L2 hit), and store them into each
 // consumer's slot.  Returns the pack checksum; cks_c[k] is the checksum of
 // what consumer k received (the read-back, after any injected fault).
-template <int U = kUnroll>
+template <int U = kUnroll, int kC = kMaxFused>
 __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ src, uint8_t *__restrict__ snap,
                                                     const uint64_t *dst, uint32_t ncons, uint32_t n, uint64_t p0,
                                                     uint32_t lane, uint32_t inject_mask, uint64_t *cks_c) {
     uint64_t acc = 0;
     bool aligned = (((uintptr_t)src | (uintptr_t)snap) & 15u) == 0;
 #pragma unroll
-    for (int k = 0; k < kMaxFused; k++)
+    for (int k = 0; k < kC; k++)
         if (k < (int)ncons) aligned &= (dst[k] & 15u) == 0;
     if (!aligned) {  // rare: word path, pack then one read-back per consumer
         acc = copy_words_bytewise<false>(src, snap, 0, n, p0, lane, false);
         __syncwarp();
 #pragma unroll
-        for (int k = 0; k < kMaxFused; k++)
+        for (int k = 0; k < kC; k++)
             if (k < (int)ncons)
                 cks_c[k] += copy_words_bytewise<true>(snap, (uint8_t *)dst[k], 0, n, p0, lane, (inject_mask >> k) & 1u);
         return acc;
@@ -262,7 +262,7 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
         }
 #endif
 #pragma unroll
-        for (int k = 0; k < kMaxFused; k++) {
+        for (int k = 0; k < kC; k++) {
             if (k >= (int)ncons) break;
 #pragma unroll
             for (int u = 0; u < U; u++) {
@@ -280,7 +280,7 @@ __device__ __forceinline__ uint64_t copy_item_fused(const uint8_t *__restrict__ 
         acc += copy_words_bytewise<false>(src, snap, nvec * 16, n, p0, lane, false);
         __syncwarp();
 #pragma unroll
-        for (int k = 0; k < kMaxFused; k++)
+        for (int k = 0; k < kC; k++)
             if (k < (int)ncons)
                 cks_c[k] += copy_words_bytewise<true>(snap, (uint8_t *)dst[k], nvec * 16, n, p0, lane,
                                                       ((inject_mask >> k) & 1u) && nvec == 0);
@@ -930,7 +930,14 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 #endif
 
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fused_kernel(const FusedArgs a) {
+#ifndef VP_FUSED1_BLOCKS
+#define VP_FUSED1_BLOCKS VP_FUSED_BLOCKS
+#endif
+// kC = the consumers compiled in: 1 (the common SYNC 1 -> 1 update: fewer
+// registers) or kMaxFused.
+template <int kC>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kC == 1 ? VP_FUSED1_BLOCKS : kFusedBlocks)
+    publish_fused_kernel(const FusedArgs a) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t nwarps = gridDim.x * kWarpsPerBlock;
     uint32_t bad = 0;
@@ -944,23 +951,26 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kFusedBlocks) publish_fus
     if (w < a.nitems) q.claim(lane);
     while (w < a.nitems) {
         const Item it = a.items[w];
-        uint64_t cptr[kMaxFused];  // only the slot address differs between the lists
+        uint64_t cptr[kC];  // only the slot address differs between the lists
         uint32_t inject = 0;
 #pragma unroll
-        for (int k = 0; k < kMaxFused; k++) {
+        for (int k = 0; k < kC; k++) {
             cptr[k] = k < (int)a.ncons ? a.cons[k].items[w].ptr : 0;
             if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
         }
-        uint64_t got[kMaxFused] = {0, 0, 0, 0};
-        const uint64_t part = warp_sum(copy_item_fused<kFusedUnroll>((const uint8_t *)it.ptr, a.packed + it.packed_off, cptr,
-                                                       a.ncons, it.nbytes, it.packed_off, lane, inject, got));
+        uint64_t got[kC];
+#pragma unroll
+        for (int k = 0; k < kC; k++) got[k] = 0;
+        const uint64_t part = warp_sum(copy_item_fused<kFusedUnroll, kC>((const uint8_t *)it.ptr, a.packed + it.packed_off,
+                                                                         cptr, a.ncons, it.nbytes, it.packed_off, lane,
+                                                                         inject, got));
         const uint64_t sealed = part + a.version * kVerMix;
         if (lane == 0) {  // no concurrent reader in this path: a plain store (grid end publishes it)
             a.iseal[w].mixed = sealed;
             a.iseal[w].version = a.version;
         }
 #pragma unroll
-        for (int k = 0; k < kMaxFused; k++) {
+        for (int k = 0; k < kC; k++) {
             if (k >= (int)a.ncons) break;
             if (warp_sum(got[k]) + a.version * kVerMix != sealed) bad |= 1u << k;
         }
@@ -1577,17 +1587,20 @@ cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
     return cudaGetLastError();
 }
 
-const void *fused_kernel_fn() { return (const void *)publish_fused_kernel; }
+const void *fused_kernel_fn(uint32_t ncons) {
+    return ncons <= 1 ? (const void *)publish_fused_kernel<1> : (const void *)publish_fused_kernel<kMaxFused>;
+}
 
-Geometry fused_geometry(const Geometry &g, int device) {
+Geometry fused_geometry(const Geometry &g, int device, uint32_t ncons) {
     // same block shape, up to kFusedBlocks resident blocks per SM
     Geometry f = g;
-    f.grid = grid_for(g.items, kWarpsPerBlock, sm_count(launch_device()), kFusedBlocks);
+    f.grid = grid_for(g.items, kWarpsPerBlock, sm_count(launch_device()), ncons <= 1 ? VP_FUSED1_BLOCKS : kFusedBlocks);
     return f;
 }
 
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
-    publish_fused_kernel<<<g.grid, g.block, 0, st>>>(a);
+    if (a.ncons <= 1) publish_fused_kernel<1><<<g.grid, g.block, 0, st>>>(a);
+    else publish_fused_kernel<kMaxFused><<<g.grid, g.block, 0, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1688,7 +1701,7 @@ cudaError_t preload_kernels() {
                          (const void *)install_verify_kernel,    install_direct_fn(0, false),
                          install_direct_fn(~0ull, false),        install_direct_fn(0, true),
                          install_direct_fn(~0ull, true),
-                         (const void *)publish_fused_kernel,     (const void *)pack_seal_tma_kernel,
+                         fused_kernel_fn(1), fused_kernel_fn(kMaxFused), (const void *)pack_seal_tma_kernel,
                          (const void *)install_verify_tma_kernel, (const void *)publish_fused_tma_kernel,
                          (const void *)view_seal_kernel,         (const void *)pack_push_kernel,
                          (const void *)pack_nvls_kernel};

@@ -713,7 +713,7 @@ static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStr
                      : (fl & VIPER_FLAG_FUSED_TMA) ? true
                      : (fl & VIPER_FLAG_NO_TMA)    ? false
                                                    : kFusedTmaDefault && p->man.s_packed <= kFusedTmaMaxBytes;
-    const Geometry fg = fused_geometry(p->geo, p->device);
+    const Geometry fg = fused_geometry(p->geo, p->device, f.ncons);
     void *args[] = {(void *)&f};
     cudaKernelNodeParams kp{};
     if (tma) {
@@ -726,7 +726,7 @@ static cudaError_t launch_fused_fast(viper_model *p, const FusedArgs &f, cudaStr
         if (no_graph) return cudaLaunchKernel(l.func, kp.gridDim, kp.blockDim, args, l.smem, st);
     } else {
         if (no_graph) return launch_fused(f, fg, st);
-        kp.func = (void *)fused_kernel_fn();
+        kp.func = (void *)fused_kernel_fn(f.ncons);
         kp.gridDim = dim3(fg.grid);
         kp.blockDim = dim3(fg.block);
     }

@@ -166,7 +166,7 @@ struct Geometry {
     int grid, block;
     uint32_t items = 0;
 };
-Geometry fused_geometry(const Geometry &g, int device);  // publish_fused_kernel's grid (own occupancy)
+Geometry fused_geometry(const Geometry &g, int device, uint32_t ncons);  // publish_fused_kernel's grid (own occupancy)
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms = 0);  // max_sms > 0: at most that many SMs
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
@@ -176,7 +176,7 @@ cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device);
 cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device, int max_sms = 0);
 cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
-const void *fused_kernel_fn();  // for the one-node launch graph (runtime.cpp)
+const void *fused_kernel_fn(uint32_t ncons);  // for the one-node launch graph (runtime.cpp)
 // A kernel launch as data (function, geometry, dynamic shared memory) for the
 // one-node launch graphs of runtime.cpp; err != cudaSuccess: not launchable.
 struct LaunchSpec {
