@@ -930,6 +930,9 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 #endif
 
+#ifndef VP_FUSED_PREFETCH
+#define VP_FUSED_PREFETCH 0  // 1: next item's descriptors loaded one item ahead (A/B)
+#endif
 #ifndef VP_FUSED1_BLOCKS
 #define VP_FUSED1_BLOCKS VP_FUSED_BLOCKS
 #endif
@@ -947,6 +950,36 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kC == 1 ? VP_FUSED1_BLOCK
     const unsigned long long prof_t0 = gtimer();
     unsigned long long prof_items = 0, prof_bytes = 0;
 #endif
+#if VP_FUSED_PREFETCH
+    // The next item is known one item ahead (its claim was issued two items
+    // ahead), so its descriptors -- the producer item and each consumer's slot
+    // address -- load while this item streams.  The first two items of a warp
+    // are static (w, w + nwarps); claims then start at 2 * nwarps.
+    unsigned int *ctr = reinterpret_cast<unsigned int *>(a.flags + 1);
+    const bool dyn = a.nitems > 2 * nwarps;
+    uint32_t wn = w + nwarps;
+    uint32_t pend = 0;
+    Item it_n{};
+    uint64_t cptr_n[kC];
+    auto load_desc = [&](uint32_t x, Item &d, uint64_t *cp) {
+        if (x >= a.nitems) return;
+        d = a.items[x];
+#pragma unroll
+        for (int k = 0; k < kC; k++) cp[k] = k < (int)a.ncons ? a.cons[k].items[x].ptr : 0;
+    };
+    load_desc(w, it_n, cptr_n);
+    while (w < a.nitems) {
+        const Item it = it_n;
+        uint64_t cptr[kC];
+#pragma unroll
+        for (int k = 0; k < kC; k++) cptr[k] = cptr_n[k];
+        if (dyn && lane == 0 && wn < a.nitems) pend = atomicAdd(ctr, 1u);  // the item after wn
+        load_desc(wn, it_n, cptr_n);
+        uint32_t inject = 0;
+#pragma unroll
+        for (int k = 0; k < kC; k++)
+            if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
+#else
     WorkQueue q(reinterpret_cast<unsigned int *>(a.flags + 1), 0, nwarps, a.nitems);  // reset by the last block
     if (w < a.nitems) q.claim(lane);
     while (w < a.nitems) {
@@ -958,6 +991,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kC == 1 ? VP_FUSED1_BLOCK
             cptr[k] = k < (int)a.ncons ? a.cons[k].items[w].ptr : 0;
             if (k < (int)a.ncons && w == a.cons[k].fault_item) inject |= 1u << k;
         }
+#endif
         uint64_t got[kC];
 #pragma unroll
         for (int k = 0; k < kC; k++) got[k] = 0;
@@ -978,8 +1012,20 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kC == 1 ? VP_FUSED1_BLOCK
         prof_items++;
         prof_bytes += it.nbytes;
 #endif
+#if VP_FUSED_PREFETCH
+        w = wn;
+        if (w < a.nitems) {
+            if (dyn) {
+                const uint32_t k2 = __shfl_sync(0xffffffffu, pend, 0);
+                wn = k2 < a.nitems - 2 * nwarps ? k2 + 2 * nwarps : a.nitems;
+            } else {
+                wn = w + nwarps;
+            }
+        }
+#else
         w = q.next(w, lane);
         if (w < a.nitems) q.claim(lane);
+#endif
     }
 #if VP_WARP_PROF
     if (lane == 0 && gw < 8192) {

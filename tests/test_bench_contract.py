@@ -112,3 +112,17 @@ def test_summarize_fanout_math_and_parity():
     assert bench.summarize_fanout([prod, bad], S)["parity_ok"] is False
     un = bench.summarize_fanout([{"unsupported": "VIPER_E_UNSUPPORTED: no multicast"}] * 2, S)
     assert "unsupported" in un
+
+
+def test_bench_fanout_codes_match_the_abi():
+    """bench.py's fan-out names map to include/viper.h's VIPER_FANOUT_* codes
+    (through the binding's constants), and the baselines never headline."""
+    import bench
+    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+    assert bench.FANOUTS["direct"] == V.FANOUT_DIRECT and bench.FANOUTS["chain"] == V.FANOUT_CHAIN
+    assert bench.FANOUTS["sa"] == V.FANOUT_SCATTER_ALLGATHER and bench.FANOUTS["nvls"] == V.FANOUT_NVLS
+    assert bench.FANOUTS["push"] == V.FANOUT_PUSH and bench.FANOUTS["nccl"] == V.FANOUT_NCCL
+    assert bench.FANOUTS["ce"] == V.FANOUT_CE and bench.FANOUTS["dram"] < 0
+    hdr = open(os.path.join(ROOT, "include", "viper.h")).read()
+    for name, code in (("NVLS", 3), ("PUSH", 4), ("NCCL", 100), ("CE", 101)):
+        assert f"VIPER_FANOUT_{name} = {code}" in hdr
