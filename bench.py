@@ -63,7 +63,9 @@ def ncu_traffic(kernel, config):
     try:
         with open(os.path.join(ROOT, "profiles", "ncu_traffic.json")) as f:
             t = json.load(f)
-        return t.get(f"{kernel}:{config}", {}).get("traffic_bytes")
+        # template instances are named "<kernel><...>:<config>"; the newest capture of the kernel wins
+        keys = [k for k in t if k.split("<")[0].split(":")[0] == kernel and k.endswith(f":{config}")]
+        return t[sorted(keys, key=lambda k: "<" in k)[-1]].get("traffic_bytes") if keys else None
     except Exception:
         return None
 
@@ -80,7 +82,7 @@ def ncu_launches(config, kernel, alg_bytes, peak):
     try:
         with open(os.path.join(ROOT, LAUNCH_LISTS[config])) as f:
             t = json.load(f)
-        k = t[kernel]
+        k = t[next(n for n in t if n.split("<")[0] == kernel)]
         lib = k["total_us"] + t.get("seal_reduce_kernel", {}).get("total_us", 0.0) * k["launches"] / max(
             1, t.get("seal_reduce_kernel", {}).get("launches", 1))
         return {"file": LAUNCH_LISTS[config], "mean_us": k["mean_us"], "share_of_library_kernels":
