@@ -1624,15 +1624,6 @@ cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st) {
     return cudaLaunchKernel(pack_fn(a.s_packed, a.sys_release), dim3(g.grid), dim3(g.block), args, 0, st);
 }
 
-cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device) {
-    if (a.nitems == 0) return cudaSuccess;
-    static std::atomic<uint64_t> opted{0};
-    const cudaError_t e = opt_in_smem(pack_seal_tma_kernel, kTmaSmem, device, opted);
-    if (e != cudaSuccess) return e;
-    pack_seal_tma_kernel<<<grid_for(a.nitems, kTmaWarps, sm_count(launch_device()), 2), kTmaWarps * 32, kTmaSmem, st>>>(a);
-    return cudaGetLastError();
-}
-
 const void *fused_kernel_fn(uint32_t ncons) {
     return ncons <= 1 ? (const void *)publish_fused_kernel<1> : (const void *)publish_fused_kernel<kMaxFused>;
 }
@@ -1647,16 +1638,6 @@ Geometry fused_geometry(const Geometry &g, int device, uint32_t ncons) {
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st) {
     if (a.ncons <= 1) publish_fused_kernel<1><<<g.grid, g.block, 0, st>>>(a);
     else publish_fused_kernel<kMaxFused><<<g.grid, g.block, 0, st>>>(a);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device, int max_sms) {
-    static std::atomic<uint64_t> opted{0};
-    const cudaError_t e = opt_in_smem(install_verify_tma_kernel, kTmaSmem, device, opted);
-    if (e != cudaSuccess) return e;
-    const int sms = sm_count(launch_device());
-    const int grid = grid_for(a.nitems, kTmaWarps, max_sms > 0 && max_sms < sms ? max_sms : sms, 2);
-    install_verify_tma_kernel<<<grid, kTmaWarps * 32, kTmaSmem, st>>>(a);
     return cudaGetLastError();
 }
 
@@ -1723,12 +1704,6 @@ LaunchSpec seal_reduce_launch(const SealReduceArgs &a) {
     l.grid = (int)((a.nchunks + 7) / 8);
     l.block = 256;
     return l;
-}
-
-cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st) {
-    if (a.nchunks == 0) return cudaSuccess;
-    seal_reduce_kernel<<<(a.nchunks + 7) / 8, 256, 0, st>>>(a);
-    return cudaGetLastError();
 }
 
 // Load every kernel of the library into the current device's context now,

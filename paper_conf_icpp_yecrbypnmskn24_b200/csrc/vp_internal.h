@@ -170,11 +170,6 @@ Geometry fused_geometry(const Geometry &g, int device, uint32_t ncons);  // publ
 Geometry pick_geometry(uint32_t nitems, int device, int max_sms = 0);  // max_sms > 0: at most that many SMs
 
 cudaError_t launch_pack(const PackArgs &a, const Geometry &g, cudaStream_t st);
-// TMA bulk-copy pack (cp.async.bulk); consumers must not be PDL-chained to it
-cudaError_t launch_pack_tma(const PackArgs &a, cudaStream_t st, int device);
-// TMA bulk-copy install: direct (no scatter-allgather / multi-producer), not PDL-chained
-cudaError_t launch_install_tma(const InstallArgs &a, cudaStream_t st, int device, int max_sms = 0);
-cudaError_t launch_seal_reduce(const SealReduceArgs &a, cudaStream_t st);
 cudaError_t launch_fused(const FusedArgs &a, const Geometry &g, cudaStream_t st);
 const void *fused_kernel_fn(uint32_t ncons);  // for the one-node launch graph (runtime.cpp)
 // A kernel launch as data (function, geometry, dynamic shared memory) for the
