@@ -281,3 +281,14 @@ def test_xproc_nvls_kernel_path_unicast(mode, early, config):
                            ["--config", config, "--mode", str(mode), "--fanout", "3", "--versions", "5"],
                            env={"VIPER_TEST_NVLS_UNICAST": "1", "VIPER_EARLY_NOTIFY": early})
     assert rc == 0 and "XPROC_RESULT errors=0" in out, out[-4000:]
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("fanout", ["sa", "push", "nvls"])
+def test_example_fanout_serve(fanout):
+    """examples/fanout_serve.py: a trainer process publishes every step, two
+    inference processes serve from the latest version and end with seals equal
+    to the producer's and logits equal to the trainer's, bit for bit (NVLS falls
+    back to direct pulls where multicast is unavailable)."""
+    rc, out = run_torchrun(3, "examples/fanout_serve.py", ["--fanout", fanout, "--steps", "20"], timeout=300)
+    assert rc == 0 and f"FANOUT_SERVE ok ({fanout})" in out, out[-4000:]
