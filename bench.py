@@ -483,6 +483,29 @@ def c5_schedule(V, G, synth, flush, gpu_row):
     return res
 
 
+def schedule_from_costs(V, costs):
+    """viper_schedule (the paper's IPP, s4.3) driven by measured update costs,
+    on the synthetic Exp3 warm-up curve and Fig. 6 time magnitudes of
+    c5_schedule: costs = {name: (t_p seconds, t_c seconds)}."""
+    import numpy as np
+    rng = np.random.default_rng(5)
+    x = np.arange(50.0)
+    warm = list(2.5 * np.exp(-0.02 * x) + 0.8 + rng.normal(0, 0.01, 50))
+    t_train, t_infer = 0.07, 0.006
+    s_iter, e_iter = 50, 2000
+    total = int((e_iter - s_iter) * t_train / t_infer)
+    out = {}
+    for nm, (t_p, t_c) in costs.items():
+        sch = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
+                         t_p=t_p, t_c=t_c, x=list(x))
+        gr = V.schedule(warm, s_iter=s_iter, e_iter=e_iter, total_infers=total, t_train=t_train, t_infer=t_infer,
+                        t_p=t_p, t_c=t_c, x=list(x), algo=V.SCHED_GREEDY)
+        out[nm] = {"t_p_s": t_p, "t_c_s": t_c, "family": ["Exp2", "Exp3", "Lin2", "Expd3"][sch["family"]],
+                   "fixed_interval": sch["best_interval"], "fixed_cil": round(sch["predicted_cil"], 3),
+                   "greedy_checkpoints": len(gr["sched"]), "greedy_cil": round(gr["predicted_cil"], 3)}
+    return out
+
+
 def torch_copy_baseline(G, synth, name, flush_buf, steps=10, warmup=3):
     """the naive state-dict copy -- one torch copy_ per tensor from
     the producer's to the consumer's parameters (no snapshot, no seal, no
@@ -1190,6 +1213,12 @@ def xproc_arm(args):
                               if ok and "latency_ms" in results.get("dram", {}) else None),
             "dram_over_gpu_how": "BASELINE configs[4]: the pinned-DRAM tier's update latency over the headline "
                                  "GPU-to-GPU fan-out, same bytes (paper context: TC1 Host-Async / GPU-Async 2.7x)",
+            "schedule": (schedule_from_costs(V, {f: (results[f]["latency_ms"] * 1e-3, 0.0) for f in (head, "dram")
+                                                 if "latency_ms" in results.get(f, {})})
+                         if ok else None),
+            "schedule_how": "viper_schedule (IPP, s4.3) per channel with t_p = the measured SYNC update latency "
+                            "(the publish returns after every consumer installed) and t_c = 0, on c5_schedule's "
+                            "synthetic Exp3 warm-up curve (BASELINE configs[4]: schedule from viper_schedule)",
             "parity_ok": h.get("parity_ok", False),
             "parity": h.get("parity"),
             "nccl_broadcast_ms": None if over else round(float(t[0]), 6),
