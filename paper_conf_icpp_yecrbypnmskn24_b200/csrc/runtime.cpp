@@ -917,12 +917,6 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     }
     // side stream: everything that only needs the finished pack
     CUDA_TRY(cudaEventRecord(p->ev_packed, st));
-    if (p->cfg.fanout == VIPER_FANOUT_NCCL) {
-        // NCCL baseline: broadcast v to the consumers' staging, AFTER ev_packed:
-        // the notification that lets them join the collective waits on it
-        viper_status s = nccl_broadcast_version(p, p->d_snap[b], p->d_iseal[b], p->rank, st);
-        if (s) return s;
-    }
     CUDA_TRY(cudaStreamWaitEvent(p->side, p->ev_packed, 0));
     if (p->xproc && !sync && !p->early_notify) {
         // remote consumers read slot b without events: name v once the pack is
@@ -969,6 +963,15 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     TRACE(4);
     if (sync && dram) launch_all();
 
+    if (p->cfg.fanout == VIPER_FANOUT_NCCL) {
+        // NCCL baseline: broadcast v to the consumers' staging.  Enqueued after
+        // ev_packed (the notification that lets the consumers join waits on it)
+        // and as the very last step before that notification, so no early
+        // error return can leave the collective waiting for consumers that
+        // were never told about v.
+        viper_status s = nccl_broadcast_version(p, p->d_snap[b], p->d_iseal[b], p->rank, st);
+        if (s) return s;
+    }
     if (p->xproc) {
         if (sync) {  // name v once the pack completed, then wait for every consumer
             viper_status s = xproc_notify(p, v, b, true, p->early_notify);
