@@ -645,9 +645,24 @@ __device__ __forceinline__ bool grid_arrive(unsigned long long *flags, uint32_t 
 
 // A seal wait should stop: the host aborted the install (abort_h) or another
 // warp of this grid already timed out (its error bit is in the completion word).
+// abort_h is host memory: a read is a PCIe round trip, so the waits below ask
+// only once per kAbortPollMask + 1 polls (about every 250 us of waiting) --
+// asked on every poll, a thousand waiting warps flooded PCIe and slowed the
+// pipelined GPT-2 XL install 40-fold (profiles/r02/pipeline_overlap.log).
+constexpr uint32_t kAbortPollMask = 255;
 __device__ __forceinline__ bool wait_aborted(const InstallArgs &a) {
-    if (a.abort_h && *a.abort_h) return true;
-    return (*(volatile unsigned long long *)a.flags >> 32) & kErrTimeout;
+    if ((*(volatile unsigned long long *)a.flags >> 32) & kErrTimeout) return true;
+    return a.abort_h && *a.abort_h;
+}
+
+// lane 0's seal spin, one step: sleep with exponential backoff (32 ns .. 1 us);
+// true when the wait must end (kItemWaitNs passed, or aborted).
+__device__ __forceinline__ bool wait_step(const InstallArgs &a, uint32_t &backoff, uint64_t &waited, uint32_t &polls) {
+    __nanosleep(backoff);
+    waited += backoff;
+    if (backoff < 1024) backoff <<= 1;
+    if ((++polls & kAbortPollMask) != 0) return false;
+    return waited > kItemWaitNs || wait_aborted(a);
 }
 
 // End of an install grid: the last block to finish publishes the result and,
@@ -741,7 +756,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
             int ok = 0;
             if (lane == 0) {
                 const ISeal *ps = a.sa_isrc[peer] + w;
-                uint32_t backoff = 64;
+                uint32_t backoff = 64, polls = 0;
                 int64_t spent = 0;
                 for (;;) {
                     if (ld_acquire_sys(&ps->version) == a.version) { ok = 1; break; }
@@ -749,8 +764,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
                     spent += backoff;
                     if (backoff < 2048) backoff <<= 1;
                     // the peer is not installing this version (skipped it or
-                    // finished without it): take the item from the producer
-                    if (spent > 20000 && *a.sa_owner_pin[peer] != a.version) break;
+                    // finished without it): take the item from the producer.
+                    // (The pin word is host memory: asked every 16th poll.)
+                    if (spent > 20000 && (++polls & 15) == 0 && *a.sa_owner_pin[peer] != a.version) break;
                     if (spent > 50000000) break;  // 50 ms: never hang, fall back
                 }
             }
@@ -766,15 +782,12 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kBlocksPerSM) install_ver
         if (rp_n && !ready(is)) release_staged();
         uint64_t expect = 0;
         if (lane == 0) {
-            uint32_t backoff = 32;
+            uint32_t backoff = 32, polls = 0;
             uint64_t waited = 0;
             while (ld_acquire_sys(&is->version) != a.version) {
-                __nanosleep(backoff);
-                waited += backoff;
-                if (backoff < 1024) backoff <<= 1;
                 // never hang on a vanished producer: give up after kItemWaitNs,
-                // at once when the host aborts, or when another warp timed out
-                if (waited > kItemWaitNs || wait_aborted(a)) {
+                // when the host aborts, or when another warp timed out
+                if (wait_step(a, backoff, waited, polls)) {
                     report_err(a.flags, kErrTimeout);
                     break;
                 }
@@ -861,13 +874,10 @@ constexpr int kIdBlocks = VP_ID_BLOCKS;  // install_direct's resident blocks per
 // lane 0: wait until item w's seal shows the version (acquire, system scope:
 // the producer may be another GPU); returns its cks.  Never hangs.
 __device__ __forceinline__ uint64_t acquire_seal(const InstallArgs &a, uint32_t w) {
-    uint32_t backoff = 32;
+    uint32_t backoff = 32, polls = 0;
     uint64_t waited = 0;
     while (ld_acquire_sys(&a.iseal[w].version) != a.version) {
-        __nanosleep(backoff);
-        waited += backoff;
-        if (backoff < 1024) backoff <<= 1;
-        if (waited > kItemWaitNs || wait_aborted(a)) {
+        if (wait_step(a, backoff, waited, polls)) {
             report_err(a.flags, kErrTimeout);
             break;
         }
