@@ -238,7 +238,8 @@ extern "C" viper_status viper_restore(const char *path, const viper_tensor *tens
         close(fd);
         return set_error(VIPER_E_INVAL, "%s: not a checkpoint of these %d tensors", path, n);
     }
-    if (cudaSetDevice(device) != cudaSuccess) {
+    DeviceGuard dg(device);
+    if (dg.err != cudaSuccess) {
         close(fd);
         return set_error(VIPER_E_CUDA, "cudaSetDevice(%d)", device);
     }

@@ -1044,7 +1044,7 @@ static void free_model(viper_model *m) {
             v.erase(std::remove(v.begin(), v.end(), m), v.end());
         }
     }
-    cudaSetDevice(m->device);
+    DeviceGuard dg(m->device);
     cudaDeviceSynchronize();
     flush_stop(m);
     if (m->rec) m->rec->active.store(0);
@@ -1299,7 +1299,8 @@ static viper_status register_impl(const char *model_name, int32_t role, const vi
         if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev <= 0)
             return set_error(VIPER_E_CUDA, "no CUDA device (there is no CPU fallback)");
         if (c.device < 0 || c.device >= ndev) return set_error(VIPER_E_INVAL, "bad device %d", c.device);
-        CUDA_TRY(cudaSetDevice(c.device));
+        DeviceGuard dg(c.device);  // until this call returns (the update thread sets its own)
+        if (dg.err != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice(%d): %s", c.device, cudaGetErrorString(dg.err));
         CUDA_TRY(preload_kernels());
         st = check_tensor_devices(tensors, n, c.device);
         if (st) return st;
@@ -1356,7 +1357,8 @@ viper_status viper_publish(viper_model *m, uint64_t version, void *cuda_stream) 
     if (!m || m->closed.load()) return set_error(VIPER_E_STATE, "model closed");
     if (m->role != VIPER_PRODUCER) return set_error(VIPER_E_STATE, "publish on a consumer");
     try {
-        if (cudaSetDevice(m->device) != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice");
+        DeviceGuard dg(m->device);
+        if (dg.err != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice");
         return producer_publish(m, version, (cudaStream_t)cuda_stream);
     } catch (const std::exception &e) {
         return set_error(VIPER_E_NOMEM, "publish: %s", e.what());
@@ -1432,7 +1434,7 @@ viper_status viper_release(viper_model *m, const viper_view *view, void *cuda_st
         m->views.erase(it);
     }
     if (cuda_stream) {
-        cudaSetDevice(m->device);
+        DeviceGuard dg(m->device);
         ReleaseCtx *c = new ReleaseCtx{m->rec, slot};
         cudaError_t e = cudaLaunchHostFunc((cudaStream_t)cuda_stream, release_host_fn, c);
         if (e != cudaSuccess) {
@@ -1518,7 +1520,8 @@ viper_status viper_view_seals(viper_model *m, const viper_view *view, void *dev_
         if (it == m->views.end() || it->second.slot != view->slot)
             return set_error(VIPER_E_STATE, "unknown or released view (ticket %llu)", (unsigned long long)view->ticket);
     }
-    CUDA_TRY(cudaSetDevice(m->device));
+    DeviceGuard dg(m->device);
+    if (dg.err != cudaSuccess) return set_error(VIPER_E_CUDA, "cudaSetDevice");
     const cudaStream_t st = (cudaStream_t)cuda_stream;
     if (m->man.nchunks) CUDA_TRY(cudaMemsetAsync(dev_seals_out, 0, sizeof(Seal) * m->man.nchunks, st));
     ViewSealArgs a{};

@@ -43,6 +43,24 @@ inline bool copy_staged(int32_t tier, int32_t f) {
 // (push: peer stores; NVLS: multicast stores).
 inline bool staged_fanout(int32_t f) { return f == VIPER_FANOUT_NVLS || f == VIPER_FANOUT_PUSH; }
 
+// A public call runs on the model's GPU and leaves the caller's current device
+// as it found it (a process driving several GPUs, e.g. torch's current device,
+// must not see it change under a publish / release / unregister).
+struct DeviceGuard {
+    int prev = -1;
+    cudaError_t err = cudaSuccess;
+    explicit DeviceGuard(int dev) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) err = cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+    DeviceGuard(const DeviceGuard &) = delete;
+    DeviceGuard &operator=(const DeviceGuard &) = delete;
+};
+
 struct alignas(64) ConsRec {
     std::atomic<uint64_t> state;         // (v << 1) | slot, 0 = nothing installed (device-written)
     std::atomic<uint64_t> pin;           // snapshot version being read, 0 = none (device-cleared)

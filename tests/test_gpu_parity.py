@@ -755,12 +755,17 @@ def test_two_gpus_in_process(mode, flags):
     prod_t = G.alloc_model(specs, device="cuda:0")
     cons_t = G.alloc_model(specs, device="cuda:1")
     name = uname()
+    torch.cuda.set_device(0)
     cons = V.Model(name, V.CONSUMER, cons_t, device=1)
+    assert torch.cuda.current_device() == 0  # public calls leave the caller's device alone
     prod = V.Model(name, V.PRODUCER, prod_t, device=0, mode=mode, flags=flags)
     try:
         for v in (1, 2, 3):
             G.fill_model(prod_t, specs, seed, v)
+            torch.cuda.set_device(1)
             prod.publish(v)
+            assert torch.cuda.current_device() == 1
+            torch.cuda.set_device(0)
             cons.wait_installed(v)
             view = cons.acquire_latest()
             assert view.version == v
@@ -768,10 +773,13 @@ def test_two_gpus_in_process(mode, flags):
             n = cons.stats()["nchunks"]
             buf = torch.empty(16 * n, dtype=torch.uint8, device="cuda:1")
             cons.view_seals(view, buf)
+            assert torch.cuda.current_device() == 0
             torch.cuda.synchronize(1)
             _, s_or, _ = oracle_packed_and_seals(specs, seed, v, 2 << 20)
             assert np.array_equal(buf.view(torch.int64).cpu().numpy().view(np.uint64).reshape(n, 2), s_or)
-            cons.release(view)
+            cons.release(view, stream=torch.cuda.current_stream(1))
+            assert torch.cuda.current_device() == 0
     finally:
         cons.close()
         prod.close()
+    assert torch.cuda.current_device() == 0
