@@ -541,7 +541,16 @@ static viper_status wait_install_bounded(viper_model *c, uint64_t v, int b) {
         // the install kernel's last block reports in the mapped status word
         // before the grid retires: the cheap, early signal (the stream query
         // below covers errors and launches that never report)
-        if (c->rec->status.load() != 1) {
+        if (const int32_t s = c->rec->status.load(); s != 1) {
+            // success: the last block stores the swap right after the status,
+            // so wait for that word instead of for the grid to retire (a
+            // stream synchronisation adds microseconds to every SYNC update;
+            // later work on this stream is ordered behind the grid anyway)
+            if (s == VIPER_OK) {
+                const int64_t ts = now_ns();
+                while ((c->rec->state.load() >> 1) != v && now_ns() - ts < 1000000000ll) cpu_relax();
+                if ((c->rec->state.load() >> 1) == v) return VIPER_OK;
+            }
             const cudaError_t e = cudaStreamSynchronize(c->ustream);
             return e == cudaSuccess ? VIPER_OK : set_error(VIPER_E_CUDA, "install: %s", cudaGetErrorString(e));
         }
@@ -804,6 +813,13 @@ static viper_status producer_publish(viper_model *p, uint64_t v, cudaStream_t st
     if (p->xproc && p->early_notify) {  // v is named when the stream reaches the pack (xproc.cpp)
         viper_status s = xproc_notify_early(p, v, b, st);
         if (s) return s;
+    } else if (p->xproc && sync && !dram) {
+        // SYNC, named only once the pack completed: wake the consumers' update
+        // threads now, so they are spinning on the published word (not asleep
+        // on the futex, tens of us to wake) when it lands.  A pack longer than
+        // their spin sends them back to sleep; the notification wakes them.
+        ctrl->pub_seq.fetch_add(1);
+        futex_wake_all(&ctrl->pub_seq);
     }
     const bool timing = p->cfg.flags & VIPER_FLAG_TIMING;
     std::vector<viper_model *> launched;
