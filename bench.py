@@ -1183,7 +1183,7 @@ def xproc_arm(args):
     if rank == 0:
         peak, peak_kind = load_peaks()
         h = results[head]
-        ok = "unsupported" not in h
+        ok = "latency_ms" in h  # (an unsupported or failed fan-out has no latency: the line still prints)
         lat_ms = h["latency_ms"] if ok else None
         inst = max(h["install_kernel_us_per_consumer"]) if ok else None
         cons = [c for c in conc_all[1:] if "unsupported" not in c]

@@ -451,11 +451,24 @@ viper_status launch_prepared(PreparedInstall &pi, const SnapSource &src, int b, 
     int launch_dev = c->device;
     cudaGetDevice(&launch_dev);  // a SYNC publish launches on the producer's GPU
     pi.a.sys_swap = launch_dev != c->device ? 1u : 0u;
+    // A pipelined install whose producer packs on this same GPU (ranks sharing
+    // a GPU with early notification forced, e.g. under MPS, where the two
+    // grids run concurrently) gets at most half of the SMs: its warps wait for
+    // items the pack has not sealed yet, and a grid holding every SM would
+    // keep the pack from ever being scheduled.
+    int max_sms = c->cfg.install_sms;
+    Geometry geo = c->geo;
+    if (!complete && c->prod_same_gpu) {
+        int sms = 148;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device);
+        max_sms = max_sms > 0 ? std::min(max_sms, std::max(1, sms / 2)) : std::max(1, sms / 2);
+        geo = pick_geometry(pi.a.nitems, c->device, max_sms);
+    }
     if (timing) CUDA_TRY(cudaEventRecord(c->ev_t[0], st));
     if (pdl && !timing && !tma)  // PDL: a plain stream launch
         CUDA_TRY(launch_install(pi.a, c->geo, st, true, use_direct, c->man.s_packed));
     else
-        CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, c->geo, tma, c->device, c->cfg.install_sms, use_direct,
+        CUDA_TRY(launch_spec(c->g_inst, install_launch(pi.a, geo, tma, c->device, max_sms, use_direct,
                                                        c->man.s_packed, !complete),
                              pi.a, st));
     if (timing) {
@@ -489,16 +502,25 @@ SnapSource source_of(const viper_model *p) {
 }
 
 // After the install kernel of v completed on the host's view of the stream.
+// v is reported done (the SYNC producer may return) BEFORE the bookkeeping:
+// under VIPER_FLAG_TIMING the kernel-time event is synchronised only after
+// that, with stats_mu held throughout, so a stats reader still sees v's
+// numbers and the timing costs the update nothing.
 viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
     ConsRec *r = c->rec;
     viper_status st = r->status.load();
     if (st == 1) st = set_error(VIPER_E_CUDA, "install kernel did not report");
-    float dev_ms = -1.f;
-    if (c->timing_pending && cudaEventSynchronize(c->ev_t[1]) == cudaSuccess &&
-        cudaEventElapsedTime(&dev_ms, c->ev_t[0], c->ev_t[1]) == cudaSuccess)
-        c->timing_pending = false;
     {
         std::lock_guard<std::mutex> lk(c->stats_mu);
+        r->pin.store(0);
+        r->last_status.store(st);
+        r->done_version.store(v);
+        r->done_seq.fetch_add(1);
+        if (r->waiters.load() > 0) futex_wake_all(&r->done_seq);
+        float dev_ms = -1.f;
+        if (c->timing_pending && cudaEventSynchronize(c->ev_t[1]) == cudaSuccess &&
+            cudaEventElapsedTime(&dev_ms, c->ev_t[0], c->ev_t[1]) == cudaSuccess)
+            c->timing_pending = false;
         if (dev_ms >= 0) c->stats.t_install_dev_us = dev_ms * 1e3;
         c->stats.last_status = st;
         c->stats.t_install_us = t_install_us;
@@ -509,12 +531,7 @@ viper_status finish_install(viper_model *c, uint64_t v, double t_install_us) {
             c->stats.failures++;
         }
     }
-    r->pin.store(0);
-    r->last_status.store(st);
     log_update("consumer", c, v, st, t_install_us, c->stats.writer_wait_us, "writer_wait_us");
-    r->done_version.store(v);
-    r->done_seq.fetch_add(1);
-    if (r->waiters.load() > 0) futex_wake_all(&r->done_seq);
     return st;
 }
 
@@ -651,6 +668,7 @@ void update_loop(viper_model *c) {
         }
         c->attempted = v;
         const int64_t tp = ctrl->pub_time_ns.load();
+        const int64_t te = ctrl->pub_entry_ns.load(std::memory_order_relaxed);
         const int64_t t0 = now_ns();
         NvtxRange nvtx("viper_install");
         viper_status st;
@@ -667,16 +685,15 @@ void update_loop(viper_model *c) {
                    : set_error(VIPER_E_STATE, "producer gone");
         }
         if (st == VIPER_OK) st = wait_install_bounded(c, v, b);
+        {
+            std::lock_guard<std::mutex> sl(c->stats_mu);
+            c->stats.t_notify_us = tp ? (t0 - tp) / 1e3 : 0.0;
+            c->stats.t_pickup_us = te ? (t0 - te) / 1e3 : 0.0;
+        }
         if (st == VIPER_OK) st = finish_install(c, v, (now_ns() - t0) / 1e3);
         else {
             r->status.store(st);
             finish_install(c, v, (now_ns() - t0) / 1e3);
-        }
-        {
-            std::lock_guard<std::mutex> sl(c->stats_mu);
-            c->stats.t_notify_us = tp ? (t0 - tp) / 1e3 : 0.0;
-            const int64_t te = ctrl->pub_entry_ns.load(std::memory_order_relaxed);
-            c->stats.t_pickup_us = te ? (t0 - te) / 1e3 : 0.0;
         }
         lk.unlock();
         fire_callback(c, v, st);

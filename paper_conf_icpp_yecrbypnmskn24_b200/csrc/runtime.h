@@ -194,6 +194,7 @@ struct viper_model {
 
     // ---------------- consumer
     int32_t cidx = -1;
+    bool prod_same_gpu = false;  // consumer (cross-process): the producer runs on this GPU too
     vp::ConsRec *rec = nullptr, *rec_dev = nullptr;
     std::vector<void *> slot_ptrs[2];
     vp::Item *d_slot_items[2] = {nullptr, nullptr};  // consumer work lists per slot

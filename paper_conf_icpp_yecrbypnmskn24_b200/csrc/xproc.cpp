@@ -470,6 +470,7 @@ viper_status xproc_register(viper_model *m, const viper_tensor *tensors, const v
         for (int r = 0; r < bs->rank; r++)
             if (all[r].role != VIPER_PRODUCER) idx++;
         m->cidx = idx;
+        m->prod_same_gpu = strncmp(pr.pci, me.pci, sizeof me.pci) == 0;
         st = open_segment(m, pr.shm_path, pr.shm_bytes);
         if (st == VIPER_OK) st = map_control(m);
         if (st == VIPER_OK && m->ctrl->magic != kCtrlMagic) st = set_error(VIPER_E_PEER, "bad control segment");
