@@ -681,10 +681,12 @@ __device__ __forceinline__ void install_finish(const InstallArgs &a, bool bad) {
         // this thread observed -- orders every block's peer stores before the
         // swap becomes visible.
         if (a.sys_swap) asm volatile("fence.acq_rel.sys;" ::: "memory");
+        // the pin first: the host takes the status / swap as "done" and may
+        // pin its next snapshot at once, which a late clear would undo
+        if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer (every block has arrived)
+        if (a.ctr) *a.ctr = 0;      // work counter: every warp stopped claiming
         if (a.status_h) *a.status_h = st;
         if (st == 0 && a.state_h) *a.state_h = (a.version << 1) | (uint64_t)a.target;  // the atomic swap
-        if (a.pin_h) *a.pin_h = 0;  // snapshot no longer read by this consumer
-        if (a.ctr) *a.ctr = 0;      // work counter: every warp stopped claiming
     }
 }
 
