@@ -4,6 +4,9 @@
 # contexts, so the cross-process engine (IPC pull, shm notification, system-
 # scope seals, the early-notified item pipeline) is timed without context
 # switches.  Still one GPU: no byte crosses NVLink.
+# Caution: under MPS a kernel can outlive a client process that a timeout
+# killed.  Only run kernels whose waits are bounded (every kernel of
+# libviper.so is), and stop the daemon (the EXIT trap) even on failure.
 mkdir -p gpurun_out
 export CUDA_MPS_PIPE_DIRECTORY=/tmp/viper_mps_pipe CUDA_MPS_LOG_DIRECTORY=/tmp/viper_mps_log
 mkdir -p $CUDA_MPS_PIPE_DIRECTORY $CUDA_MPS_LOG_DIRECTORY
