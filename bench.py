@@ -1077,6 +1077,79 @@ def xproc_concurrent(V, G, synth, name, rank, world, dev, gloo, fanout, seconds=
     return res
 
 
+def xproc_line(args, world, name, S, ndev, over, head, results, conc_all, t, e2e, clocks):
+    """Rank 0's JSON line of the N > 1 arm.  t = [NCCL broadcast ms, CE pull ms,
+    e2e ms, e2e digest failures], max over ranks.  A headline fan-out that
+    failed or was unsupported has no latency: the line still prints (value
+    null, its errors under `fanouts`)."""
+    from paper_conf_icpp_yecrbypnmskn24_b200 import viper as V
+    h = results[head]
+    ok = "latency_ms" in h  # (an unsupported or failed fan-out has no latency: the line still prints)
+    lat_ms = h["latency_ms"] if ok else None
+    inst = max(h["install_kernel_us_per_consumer"]) if ok else None
+    cons = [c for c in conc_all[1:] if "unsupported" not in c]
+    out = {
+        "metric": METRIC, "value": lat_ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": lat_ms, "higher_is_better": False, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
+        "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
+        "config": {"workload": f"{name}: 1 producer -> {world - 1} consumer(s) "
+                               f"{'sharing one GPU (code path only, no NVLink)' if over else 'over NVLink'} "
+                               f"({FANOUT_NAMES[FANOUTS[head]]}), SYNC",
+                   "baseline_config": f"BASELINE.json configs[{CONFIG_INDEX[name]}]", "fanout": head,
+                   "model_bytes": S, "devices_visible": ndev, "oversubscribed": over,
+                   "l2": "flushed on every rank before every update (256 MiB write + 256 MiB read)",
+                   "parallelism": f"1 producer + {world - 1} consumers, one process per GPU"},
+        "update_gbps_per_consumer": h.get("update_gbps_per_consumer"),
+        "roofline": None if (over or not ok) else {
+            "bound": "nvlink", "kernel": "update: pack -> NVLink delivery -> install + verify + swap (pipelined)",
+            "achieved": round(S / (lat_ms * 1e-3) / 1e9, 2), "peak": NVLINK_GBS, "unit": "GB/s",
+            "frac": round(S / (lat_ms * 1e-3) / 1e9 / NVLINK_GBS, 4), "traffic": None,
+            "peak_kind": "NVLink 5 per direction per GPU (north_star; B200_PROFILING.md)",
+            "algorithmic_bytes": S, "formula": "f_NVL = (S / L_update) / 900 GB/s (SURVEY s8(d))",
+            "install_kernel": {"us": inst, "achieved": round(S / (inst * 1e-6) / 1e9, 2) if inst else None,
+                               "frac": h["install_kernel_nvlink_frac"]}},
+        "fanouts": results,
+        "dram_over_gpu": (round(results["dram"]["latency_ms"] / lat_ms, 3)
+                          if ok and "latency_ms" in results.get("dram", {}) else None),
+        "dram_over_gpu_how": "BASELINE configs[4]: the pinned-DRAM tier's update latency over the headline "
+                             "GPU-to-GPU fan-out, same bytes (paper context: TC1 Host-Async / GPU-Async 2.7x)",
+        "schedule": (schedule_from_costs(V, {f: (results[f]["latency_ms"] * 1e-3, 0.0) for f in (head, "dram")
+                                             if "latency_ms" in results.get(f, {})})
+                     if ok else None),
+        "schedule_how": "viper_schedule (IPP, s4.3) per channel with t_p = the measured SYNC update latency "
+                        "(the publish returns after every consumer installed) and t_c = 0, on c5_schedule's "
+                        "synthetic Exp3 warm-up curve (BASELINE configs[4]: schedule from viper_schedule)",
+        "parity_ok": h.get("parity_ok", False),
+        "parity": h.get("parity"),
+        "nccl_broadcast_ms": None if over else round(float(t[0]), 6),
+        "ce_pull_ms": round(float(t[1]), 6),
+        "ce_pull_how": "SURVEY B2 baseline: every consumer pulls the producer's S bytes at once with the copy "
+                       "engine (torch copy_ from the CUDA-IPC-mapped producer buffer = cudaMemcpyPeerAsync), "
+                       "CUDA events, max over consumers",
+        "concurrent_acquire": {
+            "how": f"ASYNC publish every 2 ms for 2 s ({FANOUT_NAMES[FANOUTS[head]]}); per consumer a reader "
+                   "thread acquires, compares every weight byte with VGEN(view.version) on its GPU, releases",
+            "torn_views": sum(c["torn"] for c in cons), "version_regressions": sum(c["regress"] for c in cons),
+            "views_per_s_idle": [round(c["views_idle"], 1) for c in cons],
+            "views_per_s_during_updates": [round(c["views_busy"], 1) for c in cons],
+            "publishes": conc_all[0].get("publishes"), "installs": [c["installs"] for c in cons],
+            "errors": [e for c in conc_all for e in c.get("errors", [])][:4],
+            **({"unsupported": conc_all[0]["unsupported"]} if "unsupported" in conc_all[0] else {})},
+        "gpu_launches": (2 + (world - 1)) * args.steps,
+        "gpu_launches_how": "per update: pack (+ push / NVLS stores) and seal_reduce on the producer, one "
+                            "install per consumer",
+        "clocks": clocks,
+        "cpu_baseline": None,
+        "cpu_baseline_note": "the oracle is timed on rank 0 at N = 1 only (task rule); see the N = 1 line",
+        "e2e": {"value": round(float(t[2]), 6), "unit": "ms", "h2d_bytes_per_step": e2e["h2d"],
+                "d2h_bytes_per_step": e2e["d2h"], "digest_ok": bool(float(t[3]) == 0.0),
+                "how": "rank 0: pinned host -> device copy of the step's weights, SYNC publish (returns "
+                       "after every consumer swapped), D2H of the chunk-seal digest; host clock"},
+    }
+    return out
+
+
 def xproc_arm(args):
     """N > 1: one process per GPU (self-launched by main() when WORLD_SIZE is
     unset).  Rank 0 is the producer, ranks 1..N-1 the consumers.  The workload
@@ -1181,71 +1254,8 @@ def xproc_arm(args):
                      dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX, group=gloo)
     if rank == 0:
-        peak, peak_kind = load_peaks()
-        h = results[head]
-        ok = "latency_ms" in h  # (an unsupported or failed fan-out has no latency: the line still prints)
-        lat_ms = h["latency_ms"] if ok else None
-        inst = max(h["install_kernel_us_per_consumer"]) if ok else None
-        cons = [c for c in conc_all[1:] if "unsupported" not in c]
-        out = {
-            "metric": METRIC, "value": lat_ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": lat_ms, "higher_is_better": False, "scaling": "weak",
-            "vs_baseline": None, "dtype": "u32", "model_dtype": "f32" if name in ("ptychonn", "resnet50") else "bf16",
-            "data": "synthetic (VGEN seeded random-init parameters, BASELINE.json shapes)",
-            "config": {"workload": f"{name}: 1 producer -> {world - 1} consumer(s) "
-                                   f"{'sharing one GPU (code path only, no NVLink)' if over else 'over NVLink'} "
-                                   f"({FANOUT_NAMES[FANOUTS[head]]}), SYNC",
-                       "baseline_config": f"BASELINE.json configs[{CONFIG_INDEX[name]}]", "fanout": head,
-                       "model_bytes": S, "devices_visible": ndev, "oversubscribed": over,
-                       "l2": "flushed on every rank before every update (256 MiB write + 256 MiB read)",
-                       "parallelism": f"1 producer + {world - 1} consumers, one process per GPU"},
-            "update_gbps_per_consumer": h.get("update_gbps_per_consumer"),
-            "roofline": None if (over or not ok) else {
-                "bound": "nvlink", "kernel": "update: pack -> NVLink delivery -> install + verify + swap (pipelined)",
-                "achieved": round(S / (lat_ms * 1e-3) / 1e9, 2), "peak": NVLINK_GBS, "unit": "GB/s",
-                "frac": round(S / (lat_ms * 1e-3) / 1e9 / NVLINK_GBS, 4), "traffic": None,
-                "peak_kind": "NVLink 5 per direction per GPU (north_star; B200_PROFILING.md)",
-                "algorithmic_bytes": S, "formula": "f_NVL = (S / L_update) / 900 GB/s (SURVEY s8(d))",
-                "install_kernel": {"us": inst, "achieved": round(S / (inst * 1e-6) / 1e9, 2) if inst else None,
-                                   "frac": h["install_kernel_nvlink_frac"]}},
-            "fanouts": results,
-            "dram_over_gpu": (round(results["dram"]["latency_ms"] / lat_ms, 3)
-                              if ok and "latency_ms" in results.get("dram", {}) else None),
-            "dram_over_gpu_how": "BASELINE configs[4]: the pinned-DRAM tier's update latency over the headline "
-                                 "GPU-to-GPU fan-out, same bytes (paper context: TC1 Host-Async / GPU-Async 2.7x)",
-            "schedule": (schedule_from_costs(V, {f: (results[f]["latency_ms"] * 1e-3, 0.0) for f in (head, "dram")
-                                                 if "latency_ms" in results.get(f, {})})
-                         if ok else None),
-            "schedule_how": "viper_schedule (IPP, s4.3) per channel with t_p = the measured SYNC update latency "
-                            "(the publish returns after every consumer installed) and t_c = 0, on c5_schedule's "
-                            "synthetic Exp3 warm-up curve (BASELINE configs[4]: schedule from viper_schedule)",
-            "parity_ok": h.get("parity_ok", False),
-            "parity": h.get("parity"),
-            "nccl_broadcast_ms": None if over else round(float(t[0]), 6),
-            "ce_pull_ms": round(float(t[1]), 6),
-            "ce_pull_how": "SURVEY B2 baseline: every consumer pulls the producer's S bytes at once with the copy "
-                           "engine (torch copy_ from the CUDA-IPC-mapped producer buffer = cudaMemcpyPeerAsync), "
-                           "CUDA events, max over consumers",
-            "concurrent_acquire": {
-                "how": f"ASYNC publish every 2 ms for 2 s ({FANOUT_NAMES[FANOUTS[head]]}); per consumer a reader "
-                       "thread acquires, compares every weight byte with VGEN(view.version) on its GPU, releases",
-                "torn_views": sum(c["torn"] for c in cons), "version_regressions": sum(c["regress"] for c in cons),
-                "views_per_s_idle": [round(c["views_idle"], 1) for c in cons],
-                "views_per_s_during_updates": [round(c["views_busy"], 1) for c in cons],
-                "publishes": conc_all[0].get("publishes"), "installs": [c["installs"] for c in cons],
-                "errors": [e for c in conc_all for e in c.get("errors", [])][:4],
-                **({"unsupported": conc_all[0]["unsupported"]} if "unsupported" in conc_all[0] else {})},
-            "gpu_launches": (2 + (world - 1)) * args.steps,
-            "gpu_launches_how": "per update: pack (+ push / NVLS stores) and seal_reduce on the producer, one "
-                                "install per consumer",
-            "clocks": clk.summary(),
-            "cpu_baseline": None,
-            "cpu_baseline_note": "the oracle is timed on rank 0 at N = 1 only (task rule); see the N = 1 line",
-            "e2e": {"value": round(float(t[2]), 6), "unit": "ms", "h2d_bytes_per_step": e2e["h2d"],
-                    "d2h_bytes_per_step": e2e["d2h"], "digest_ok": bool(float(t[3]) == 0.0),
-                    "how": "rank 0: pinned host -> device copy of the step's weights, SYNC publish (returns "
-                           "after every consumer swapped), D2H of the chunk-seal digest; host clock"},
-        }
+        out = xproc_line(args, world, name, S, ndev, over, head, results, conc_all, [float(x) for x in t], e2e,
+                         clk.summary())
         print(json.dumps(out), flush=True)
     dist.barrier(group=gloo)
     dist.destroy_process_group()

@@ -114,6 +114,39 @@ def test_summarize_fanout_math_and_parity():
     assert "unsupported" in un
 
 
+def test_xproc_line_survives_a_failed_headline():
+    """The N > 1 line prints even when the headline fan-out failed (it once
+    raised KeyError and lost the line): value null, no roofline, the error
+    kept under `fanouts`; with a verified headline, value = its latency and
+    the NVLink fraction follows from it."""
+    import types
+
+    import bench
+    S = 102228128
+    args = types.SimpleNamespace(steps=3, warmup=3)
+    conc = [{"publishes": 10}, {"torn": 0, "regress": 0, "views_idle": 100.0, "views_busy": 90.0, "installs": 10}]
+    e2e = {"h2d": S, "d2h": 784}
+    t = [0.5, 0.4, 2.0, 0.0]
+    clocks = {"sm_mhz": 1965.0, "sm_max_mhz": 1965.0, "reasons": []}
+    failed = bench.summarize_fanout([{"lat": [], "host": [], "inst": [], "errors": ["publish(1): VIPER_E_TIMEOUT"],
+                                      "verify": {}, "s_packed": S}, {"lat": [], "host": [], "inst": [], "errors": [],
+                                                                     "verify": {}, "s_packed": S}], S)
+    line = bench.xproc_line(args, 2, "resnet50", S, 2, False, "direct", {"direct": failed}, conc, t, e2e, clocks)
+    json.dumps(line)
+    assert line["value"] is None and line["roofline"] is None and line["parity_ok"] is False
+    assert line["fanouts"]["direct"]["error"] and line["n_gpus"] == 2
+    ver_ok = {"seals_ok": True, "bytes_ok": True, "chunks": 49, "version": 7, "version_ok": True}
+    good = bench.summarize_fanout([{"lat": [0.15] * 3, "host": [0.16] * 3, "inst": [], "s_packed": S,
+                                    "verify": dict(ver_ok, bytes_ok=None)},
+                                   {"lat": [], "host": [], "inst": [120.0] * 3, "verify": ver_ok, "s_packed": S}], S)
+    line = bench.xproc_line(args, 2, "resnet50", S, 2, False, "direct", {"direct": good, "dram": failed}, conc, t,
+                            e2e, clocks)
+    json.dumps(line)
+    assert abs(line["value"] - 0.15) < 1e-12 and line["parity_ok"] is True
+    assert abs(line["roofline"]["frac"] - S / 0.15e-3 / 1e9 / 900.0) < 1e-3
+    assert line["dram_over_gpu"] is None and line["concurrent_acquire"]["torn_views"] == 0
+
+
 def test_bench_fanout_codes_match_the_abi():
     """bench.py's fan-out names map to include/viper.h's VIPER_FANOUT_* codes
     (through the binding's constants), and the baselines never headline."""
