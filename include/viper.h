@@ -25,6 +25,8 @@
  *     (NULL = the legacy default stream).
  *   - There is no CPU fallback: without a usable sm_100 device every call
  *     that needs the GPU returns VIPER_E_CUDA.
+ *   - A call that works on the model's GPU switches to it and restores the
+ *     calling thread's current CUDA device before it returns.
  */
 #ifndef VIPER_H
 #define VIPER_H
